@@ -6,6 +6,7 @@ from here and nowhere else.
 """
 from .gen import (  # noqa: F401
     CONFIGS,
+    SHAPES,
     er_bipartite,
     chung_lu_bipartite,
     planted_blocks,
