@@ -1,0 +1,148 @@
+/* gmbe.h -- C ABI of the B200 (sm_100a) maximal-biclique-enumeration library (libgmbe.so).
+ *
+ * The operation (PAPER.md = Pan et al., SC'23, cited P:<line>):
+ *   Given a bipartite graph G(U, V, E), enumerate all maximal bicliques:
+ *   pairs (L, R), L ⊆ U, R ⊆ V, both non-empty, every u∈L adjacent to every v∈R, and no biclique
+ *   (L', R') with L ∪ R ⊂ L' ∪ R'.  The library returns their number and an
+ *   order-independent 64-bit checksum, and optionally writes the pairs.
+ *   The search is the set-enumeration tree of Alg 1/2 with an explicit
+ *   excluded set Q for the maximality check, Alg 3 root tasks, pro-active pruning by
+ *   local neighbourhood size (Thm 4.1) and load-aware task splitting (Alg 4,
+ *   P:930-1010), run by a persistent CUDA kernel.
+ *
+ * Conventions (all calls):
+ *   - Return 0 (GMBE_OK) on success, a negative GMBE_E* code otherwise; gmbe_last_error() gives a
+ *     thread-local message for the last failing call on this thread.
+ *   - All ids are the CALLER's original 0-based ids and roles, in every output and in the
+ *     checksum, even when the library internally swaps U and V (it takes V := the side with fewer
+ *     vertices; on a tie the caller's orientation is kept).
+ *   - Duplicate (u, v) pairs collapse to one edge.  Isolated vertices are in no
+ *     biclique.  An empty graph enumerates to count 0, checksum 0.
+ *   - The library never takes ownership of caller memory; it copies what it needs.
+ */
+#ifndef GMBE_H_
+#define GMBE_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  GMBE_OK = 0,
+  GMBE_EINVAL = -1,       /* bad argument: NULL pointer, id >= n_u / n_v, bad option value */
+  GMBE_ENOMEM = -2,       /* device allocation failed (nothing leaks, the graph stays valid) */
+  GMBE_ECUDA = -3,        /* a CUDA runtime call or kernel failed */
+  GMBE_EUNSUPPORTED = -4, /* input beyond implemented limits (n_edges >= 2^32, ids >= 2^31) */
+  GMBE_EINTERNAL = -5     /* a device-side capacity was exceeded (workspace too small) */
+};
+
+enum { GMBE_ORDER_DEGREE = 0 /* ascending degree, ties by id */,
+       GMBE_ORDER_IDENTITY = 1 /* vertex id order; reproduces Fig 2 / Fig 5 */ };
+
+typedef struct gmbe_graph gmbe_graph; /* opaque, owned by the library */
+
+/* Options of gmbe_load_bipartite.  NULL = defaults.  Zero-initialised fields mean defaults. */
+typedef struct {
+  uint32_t struct_size;     /* sizeof(gmbe_load_opts) */
+  int32_t device;           /* CUDA device ordinal, or -1 = the current device (opts == NULL) */
+  void* cuda_stream;        /* cudaStream_t used for the build; NULL = library-owned stream */
+  uint32_t edges_on_device; /* 1: edges_uv is a device pointer (e.g. torch int32 data_ptr()) */
+  uint32_t order;           /* GMBE_ORDER_* */
+} gmbe_load_opts;
+
+/* Build the device-resident graph (steps a1-a2 of DESIGN.md): edge ingest, dedupe, orientation,
+ * degree ordering, both-side CSR, degree / 2-hop bounds and the hash tables of the checksum.
+ *   n_u, n_v   : sizes of the caller's vertex sets U and V (ids must be < n_u / < n_v)
+ *   edges_uv   : n_edges (u, v) pairs, interleaved uint32 [u0, v0, u1, v1, ...]; host memory, or
+ *                device memory if opts->edges_on_device.  Read during the call only.
+ *   out        : receives the new graph handle (free with gmbe_free_graph).
+ * Errors: EINVAL (NULL out, NULL edges with n_edges>0, id out of range), EUNSUPPORTED
+ * (n_edges >= 2^32 or n_u, n_v >= 2^31), ENOMEM, ECUDA. */
+int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* edges_uv, uint64_t n_edges,
+                        const gmbe_load_opts* opts, gmbe_graph** out);
+
+typedef struct {
+  uint64_t n_u, n_v;         /* caller's sizes */
+  uint64_t n_edges_unique;   /* |E| after dedupe */
+  uint32_t delta_u, delta_v; /* Δ(U), Δ(V) in the library's orientation (V = smaller side) */
+  uint32_t wedge_bound_v;    /* max_v Σ_{u∈N(v)} |N(u)|  (> Δ2(V)) */
+  uint32_t swapped;          /* 1 if the library's U is the caller's V */
+  uint32_t order;            /* GMBE_ORDER_* used at load */
+  uint32_t device;
+} gmbe_graph_info;
+
+int gmbe_graph_info_get(const gmbe_graph* g, gmbe_graph_info* out);
+void gmbe_free_graph(gmbe_graph* g); /* NULL-safe */
+
+/* Paper's node_buf bound (Sec 4.1): (3·Δ(V) + 2·Δ2(V)) · sizeof(int) bytes per
+ * subtree procedure -- e.g. BookCrossing 13,601 / 53,915 -> 594,532 B ("595 KB").
+ * Pure function, no device needed. */
+uint64_t gmbe_node_buf_bound_bytes(uint64_t delta_v, uint64_t delta2_v);
+/* Paper's per-subtree size without node reuse (Sec 3.1): Δ(V)·(Δ(V)+Δ2(V))·4 B. */
+uint64_t gmbe_naive_alloc_bytes(uint64_t delta_v, uint64_t delta2_v);
+
+/* Options of gmbe_enumerate.  NULL = defaults; zero-initialised fields mean the default noted. */
+typedef struct {
+  uint32_t struct_size;   /* sizeof(gmbe_opts); 0 = treat the struct as all-defaults */
+  uint32_t no_prune;      /* 1 disables Thm 4.1 pruning (GMBE-W/O_PRUNE ablation) */
+  uint32_t no_split;      /* 1 disables load-aware splitting (Alg 4 L17-26) */
+  uint32_t bound_height;  /* split if min(|L|,|C|) > bound_height ...   (default 20) */
+  uint32_t bound_size;    /* ... and min(|L|,|C|)·|C| > bound_size       (default 1500) */
+  uint32_t warps_per_sm;  /* resident warps per SM of the persistent kernel (0 = auto) */
+  uint32_t part_index;    /* root shard: enumerate the roots whose degree rank r satisfies */
+  uint32_t part_count;    /*   r % part_count == part_index (0 = 1 part); shards partition the
+                               output, so counts / checksums add (mod 2^64) across parts */
+  uint32_t counters;      /* 1: also compute nodes/nonmax-exact algo_bytes (slower; no early
+                               exit in the maximality scan).  nodes / nonmax are always exact. */
+  uint32_t reserved0;
+  /* Optional bounded output (device-accessible memory: device or mapped pinned host).
+   * Record = [|L|, |R|, L ids (caller U ids), R ids (caller V ids)], order within a record and of
+   * records unspecified; out_offsets[i] = word offset of record i in out_ids.  A full buffer is
+   * not an error: result.truncated = 1 while count / checksum stay complete; a record that did
+   * not fit has out_offsets[i] = UINT64_MAX when i < out_offsets_cap. */
+  uint64_t* out_offsets;
+  uint64_t out_offsets_cap;
+  uint32_t* out_ids;
+  uint64_t out_ids_cap;
+  /* Optional per-root counts (HOST memory, length = library-internal |V|): bicliques emitted under
+   * each root vertex, indexed by the root's caller id on the library's V side. */
+  uint64_t* per_root_count;
+  /* Workspace (0 = auto): words of the per-warp node stack arena; words / number of task slabs. */
+  uint64_t arena_words;
+  uint64_t slab_words;
+  uint64_t n_slabs;
+  void* cuda_stream;      /* NULL = the graph's stream */
+} gmbe_opts;
+
+typedef struct {
+  uint64_t count;         /* maximal bicliques enumerated (this shard) */
+  uint64_t checksum;      /* Σ h(L,R) mod 2^64 (this shard) */
+  uint64_t n_written;     /* records written to the output buffer */
+  uint64_t truncated;     /* 1 if the output buffer was too small */
+  uint64_t roots_run;     /* roots not skipped by the Alg 3 L7 check */
+  uint64_t nodes;         /* generated, unpruned child nodes (canonical tree; roots excluded) */
+  uint64_t nonmax;        /* nodes failing the maximality check */
+  uint64_t algo_bytes;    /* DESIGN.md algorithmic bytes (only if opts.counters) */
+  uint64_t algo_bytes_qfull;
+  uint64_t splits;        /* nodes expanded in split mode */
+  uint64_t tasks;         /* subtasks enqueued */
+  double kernel_ms;       /* device time of the enumeration kernel (CUDA events) */
+} gmbe_result;
+
+/* Enumerate all maximal bicliques of g (or of one root shard).  Synchronous: returns after the
+ * result is on the host.  Concurrent calls on one graph must use distinct streams.
+ * Errors: EINVAL (NULL g/out, part_index >= part_count), ENOMEM, ECUDA, EINTERNAL. */
+int gmbe_enumerate(const gmbe_graph* g, const gmbe_opts* opts, gmbe_result* out);
+
+/* Free the device workspace (node-stack arenas, task slabs) cached on g by gmbe_enumerate.
+ * Optional: gmbe_free_graph releases it too.  NULL-safe. */
+void gmbe_release_workspace(const gmbe_graph* g);
+
+const char* gmbe_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GMBE_H_ */

@@ -1,0 +1,238 @@
+"""Python binding of libgmbe.so -- the B200 (sm_100a) maximal biclique enumeration library.
+
+Argument marshalling only: every step of the path (graph build, root generation, search,
+splitting, reduction) runs in the CUDA kernels behind the C ABI declared in include/gmbe.h.
+There is no CPU fallback: importing this package fails loudly if libgmbe.so is missing.
+
+    import paper_conf_sc_panhlzwc23_b200 as gmbe
+    g = gmbe.load(n_u, n_v, edges)          # edges: uint32 [m, 2] numpy (host) or torch (cuda)
+    r = g.enumerate()                        # -> Result(count, checksum, ...)
+"""
+import ctypes
+import os
+from dataclasses import dataclass, field
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgmbe.so")
+if not os.path.exists(LIB_PATH):
+    raise ImportError("libgmbe.so is not built (run `python -c 'import __graft_entry__ as e; e.build()'`); "
+                      "there is no CPU fallback")
+_lib = ctypes.CDLL(LIB_PATH)
+
+GMBE_OK, GMBE_EINVAL, GMBE_ENOMEM, GMBE_ECUDA, GMBE_EUNSUPPORTED, GMBE_EINTERNAL = 0, -1, -2, -3, -4, -5
+ORDER = {"degree": 0, "identity": 1}
+EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmbe_node_buf_bound_bytes",
+           "gmbe_naive_alloc_bytes", "gmbe_enumerate", "gmbe_release_workspace", "gmbe_last_error")
+
+_u32, _i32, _u64, _vp = ctypes.c_uint32, ctypes.c_int32, ctypes.c_uint64, ctypes.c_void_p
+
+
+class LoadOpts(ctypes.Structure):
+    _fields_ = [("struct_size", _u32), ("device", _i32), ("cuda_stream", _vp),
+                ("edges_on_device", _u32), ("order", _u32)]
+
+
+class GraphInfo(ctypes.Structure):
+    _fields_ = [("n_u", _u64), ("n_v", _u64), ("n_edges_unique", _u64), ("delta_u", _u32),
+                ("delta_v", _u32), ("wedge_bound_v", _u32), ("swapped", _u32), ("order", _u32),
+                ("device", _u32)]
+
+
+class Opts(ctypes.Structure):
+    _fields_ = [("struct_size", _u32), ("no_prune", _u32), ("no_split", _u32), ("bound_height", _u32),
+                ("bound_size", _u32), ("warps_per_sm", _u32), ("part_index", _u32),
+                ("part_count", _u32), ("counters", _u32), ("reserved0", _u32),
+                ("out_offsets", _vp), ("out_offsets_cap", _u64), ("out_ids", _vp),
+                ("out_ids_cap", _u64), ("per_root_count", _vp), ("arena_words", _u64),
+                ("slab_words", _u64), ("n_slabs", _u64), ("cuda_stream", _vp)]
+
+
+class CResult(ctypes.Structure):
+    _fields_ = [(n, _u64) for n in ("count", "checksum", "n_written", "truncated", "roots_run",
+                                     "nodes", "nonmax", "algo_bytes", "algo_bytes_qfull", "splits",
+                                     "tasks")] + [("kernel_ms", ctypes.c_double)]
+
+
+_lib.gmbe_load_bipartite.argtypes = [_u32, _u32, _vp, _u64, ctypes.POINTER(LoadOpts), ctypes.POINTER(_vp)]
+_lib.gmbe_load_bipartite.restype = ctypes.c_int
+_lib.gmbe_graph_info_get.argtypes = [_vp, ctypes.POINTER(GraphInfo)]
+_lib.gmbe_graph_info_get.restype = ctypes.c_int
+_lib.gmbe_free_graph.argtypes = [_vp]
+_lib.gmbe_free_graph.restype = None
+_lib.gmbe_release_workspace.argtypes = [_vp]
+_lib.gmbe_release_workspace.restype = None
+_lib.gmbe_node_buf_bound_bytes.argtypes = [_u64, _u64]
+_lib.gmbe_node_buf_bound_bytes.restype = _u64
+_lib.gmbe_naive_alloc_bytes.argtypes = [_u64, _u64]
+_lib.gmbe_naive_alloc_bytes.restype = _u64
+_lib.gmbe_enumerate.argtypes = [_vp, ctypes.POINTER(Opts), ctypes.POINTER(CResult)]
+_lib.gmbe_enumerate.restype = ctypes.c_int
+_lib.gmbe_last_error.argtypes = []
+_lib.gmbe_last_error.restype = ctypes.c_char_p
+
+
+class GmbeError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__("%s (code %d)" % (msg, code))
+        self.code = code
+
+
+def _check(rc):
+    if rc != GMBE_OK:
+        raise GmbeError(rc, _lib.gmbe_last_error().decode(errors="replace"))
+
+
+def node_buf_bound_bytes(delta_v, delta2_v):
+    """Paper's per-procedure node_buf bound (3Δ(V)+2Δ2(V))·4 B."""
+    return int(_lib.gmbe_node_buf_bound_bytes(delta_v, delta2_v))
+
+
+def naive_alloc_bytes(delta_v, delta2_v):
+    """Paper's per-subtree allocation without node reuse Δ(V)(Δ(V)+Δ2(V))·4 B."""
+    return int(_lib.gmbe_naive_alloc_bytes(delta_v, delta2_v))
+
+
+@dataclass
+class Result:
+    count: int
+    checksum: int
+    n_written: int
+    truncated: int
+    roots_run: int
+    nodes: int
+    nonmax: int
+    algo_bytes: int
+    algo_bytes_qfull: int
+    splits: int
+    tasks: int
+    kernel_ms: float
+    bicliques: list = field(default=None, repr=False)
+    per_root_count: np.ndarray = field(default=None, repr=False)
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        return None
+    return int(getattr(stream, "cuda_stream", stream))
+
+
+class Graph:
+    """Device-resident bipartite graph (opaque gmbe_graph handle)."""
+
+    def __init__(self, handle):
+        self._h = handle
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self):
+        gi = GraphInfo()
+        _check(_lib.gmbe_graph_info_get(self._h, ctypes.byref(gi)))
+        return {k: getattr(gi, k) for k, _ in GraphInfo._fields_}
+
+    def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
+                  part=(0, 1), counters=False, records=False, rec_cap=1 << 16, ids_cap=1 << 22,
+                  per_root=False, arena_words=0, slab_words=0, n_slabs=0, stream=None):
+        """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
+        o = Opts()
+        o.struct_size = ctypes.sizeof(Opts)
+        o.no_prune = 0 if prune else 1
+        o.no_split = 0 if split else 1
+        o.bound_height, o.bound_size, o.warps_per_sm = bound_height, bound_size, warps_per_sm
+        o.part_index, o.part_count = part
+        o.counters = 1 if counters else 0
+        o.arena_words, o.slab_words, o.n_slabs = arena_words, slab_words, n_slabs
+        o.cuda_stream = _stream_ptr(stream)
+        bufs = None
+        if records:
+            import torch
+            dev = torch.device("cuda", self.info()["device"])
+            offs = torch.empty(rec_cap, dtype=torch.int64, device=dev)
+            ids = torch.empty(ids_cap, dtype=torch.int32, device=dev)
+            o.out_offsets, o.out_offsets_cap = offs.data_ptr(), rec_cap
+            o.out_ids, o.out_ids_cap = ids.data_ptr(), ids_cap
+            bufs = (offs, ids)
+        prc = None
+        if per_root:
+            inf = self.info()
+            nv_int = inf["n_u"] if inf["swapped"] else inf["n_v"]
+            prc = np.zeros(max(nv_int, 1), np.uint64)
+            o.per_root_count = prc.ctypes.data
+        cr = CResult()
+        _check(_lib.gmbe_enumerate(self._h, ctypes.byref(o), ctypes.byref(cr)))
+        res = Result(**{k: getattr(cr, k) for k, _ in CResult._fields_})
+        if records:
+            offs = bufs[0][: res.n_written].cpu().numpy().view(np.uint64)
+            ids = bufs[1].cpu().numpy().view(np.uint32)
+            res.bicliques = decode_records(offs, ids)
+        if per_root:
+            res.per_root_count = prc[: (self.info()["n_u"] if self.info()["swapped"] else self.info()["n_v"])]
+        return res
+
+    def release_workspace(self):
+        if self._h:
+            _lib.gmbe_release_workspace(self._h)
+
+    def free(self):
+        if self._h:
+            _lib.gmbe_free_graph(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def decode_records(offsets, ids):
+    """Records [|L|, |R|, L ids, R ids] (caller roles) -> sorted list of (tuple(L), tuple(R)).
+    Records that did not fit (offset == UINT64_MAX) are skipped."""
+    out = []
+    for o in offsets.tolist():
+        if o == 0xFFFFFFFFFFFFFFFF:
+            continue
+        nl, nr = int(ids[o]), int(ids[o + 1])
+        out.append((tuple(sorted(ids[o + 2:o + 2 + nl].tolist())),
+                    tuple(sorted(ids[o + 2 + nl:o + 2 + nl + nr].tolist()))))
+    return sorted(out)
+
+
+def load(n_u, n_v, edges, order="degree", device=None, stream=None):
+    """gmbe_load_bipartite.  `edges`: uint32/int32 [m, 2] rows (u, v) -- numpy (host) or a CUDA
+    torch tensor (device pointer, no host copy)."""
+    lo = LoadOpts()
+    lo.struct_size = ctypes.sizeof(LoadOpts)
+    lo.device = -1 if device is None else int(device)
+    lo.cuda_stream = _stream_ptr(stream)
+    lo.order = ORDER[order]
+    keep = None
+    if hasattr(edges, "is_cuda") and edges.is_cuda:
+        e = edges.contiguous()
+        assert e.element_size() == 4
+        ptr, m = e.data_ptr(), e.numel() // 2
+        lo.edges_on_device = 1
+        if device is None:
+            lo.device = e.device.index
+        keep = e
+    else:
+        e = np.ascontiguousarray(np.asarray(edges).astype(np.uint32, copy=False).reshape(-1, 2))
+        ptr, m = (e.ctypes.data if len(e) else None), len(e)
+        keep = e
+    h = _vp()
+    _check(_lib.gmbe_load_bipartite(n_u, n_v, ptr, m, ctypes.byref(lo), ctypes.byref(h)))
+    del keep
+    return Graph(h.value)
+
+
+def enumerate_bicliques(n_u, n_v, edges, **kw):
+    """Convenience: load + enumerate + free."""
+    order = kw.pop("order", "degree")
+    g = load(n_u, n_v, edges, order=order)
+    try:
+        return g.enumerate(**kw)
+    finally:
+        g.free()

@@ -1,0 +1,349 @@
+// gmbe_graph.cu -- device graph build (DESIGN.md steps a1-a2; Sec 5 "Pre-processing",
+// P:1014-1025, and multi-edge removal).
+//
+//   a1  edge ingest -> validate ids -> orient (V := smaller side) -> pack (u<<32|v)
+//       -> radix sort -> unique (dedupe)
+//   a2  degrees -> global vertex order (ascending degree, ties by id)
+//       -> CSR of V by rank (u ascending) and CSR of U (ranks ascending) -> Δ(U), Δ(V), wedge
+//       bound (>= Δ2(V)) -> per-rank checksum hash table.
+// Sorting / scanning / selection use CUB (library primitives); everything else is our kernels.
+#include <cub/cub.cuh>
+
+#include <vector>
+
+#include "gmbe_internal.cuh"
+
+namespace {
+
+__global__ void k_pack_edges(const uint32_t* __restrict__ e, uint64_t m, uint32_t n_u, uint32_t n_v,
+                             uint32_t swapped, unsigned long long* __restrict__ keys,
+                             int* __restrict__ bad) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t u = e[2 * i], v = e[2 * i + 1];
+    if (u >= n_u || v >= n_v) {
+      *bad = 1;
+      u = 0;
+      v = 0;
+    }
+    if (swapped) {
+      uint32_t t = u;
+      u = v;
+      v = t;
+    }
+    keys[i] = ((unsigned long long)u << 32) | v;
+  }
+}
+
+__global__ void k_degrees(const unsigned long long* __restrict__ keys, uint64_t m,
+                          uint32_t* __restrict__ deg_u, uint32_t* __restrict__ deg_v) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    unsigned long long k = keys[i];
+    atomicAdd(&deg_u[k >> 32], 1u);
+    atomicAdd(&deg_v[(uint32_t)k], 1u);
+  }
+}
+
+__global__ void k_order_keys(const uint32_t* __restrict__ deg_v, uint32_t n_v, uint32_t identity,
+                             unsigned long long* __restrict__ out) {
+  for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n_v; v += gridDim.x * blockDim.x)
+    out[v] = identity ? (unsigned long long)v : (((unsigned long long)deg_v[v] << 32) | v);
+}
+
+__global__ void k_rank_maps(const unsigned long long* __restrict__ sorted, uint32_t n_v,
+                            uint32_t side_v, uint32_t* __restrict__ rank2id,
+                            uint32_t* __restrict__ id2rank, const uint32_t* __restrict__ deg_v,
+                            uint32_t* __restrict__ deg_by_rank, unsigned long long* __restrict__ hv) {
+  for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < n_v; r += gridDim.x * blockDim.x) {
+    uint32_t id = (uint32_t)sorted[r];
+    rank2id[r] = id;
+    id2rank[id] = r;
+    deg_by_rank[r] = deg_v[id];
+    hv[r] = gmbe_hid(id, side_v);
+  }
+}
+
+__global__ void k_rekey(const unsigned long long* __restrict__ keys, uint64_t m,
+                        const uint32_t* __restrict__ id2rank, unsigned long long* __restrict__ kv,
+                        unsigned long long* __restrict__ ku) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    unsigned long long k = keys[i];
+    uint32_t u = (uint32_t)(k >> 32), r = id2rank[(uint32_t)k];
+    kv[i] = ((unsigned long long)r << 32) | u;
+    ku[i] = ((unsigned long long)u << 32) | r;
+  }
+}
+
+__global__ void k_low32(const unsigned long long* __restrict__ k, uint64_t m, uint32_t* __restrict__ out) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
+       i += (uint64_t)gridDim.x * blockDim.x)
+    out[i] = (uint32_t)k[i];
+}
+
+// one warp per V rank: wedge count Σ_{u∈N(v)} |N(u)| and the maxima.
+__global__ void k_bounds(const uint32_t* __restrict__ off_v, const uint32_t* __restrict__ adj_v,
+                         const uint32_t* __restrict__ off_u, uint32_t n_v, uint32_t n_u,
+                         uint32_t* __restrict__ maxes /* [0]=Δ(V) [1]=Δ(U) [2]=wedge bound */) {
+  uint32_t lane = threadIdx.x & 31;
+  uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t r = warp; r < n_v; r += nw) {
+    uint32_t b = off_v[r], e = off_v[r + 1];
+    unsigned long long s = 0;
+    for (uint32_t i = b + lane; i < e; i += 32) {
+      uint32_t u = adj_v[i];
+      s += off_u[u + 1] - off_u[u];
+    }
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(GMBE_FULL, s, o);
+    if (lane == 0) {
+      atomicMax(&maxes[0], e - b);
+      atomicMax(&maxes[2], (uint32_t)(s > 0xffffffffull ? 0xffffffffull : s));
+    }
+  }
+  for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < n_u; u += gridDim.x * blockDim.x)
+    atomicMax(&maxes[1], off_u[u + 1] - off_u[u]);
+}
+
+struct Tmp {
+  std::vector<void*> p;
+  ~Tmp() {
+    for (void* x : p) cudaFree(x);
+  }
+  template <class T>
+  cudaError_t alloc(T** out, size_t n) {
+    void* q = nullptr;
+    cudaError_t e = cudaMalloc(&q, n ? n * sizeof(T) : 16);
+    if (e == cudaSuccess) p.push_back(q);
+    *out = (T*)q;
+    return e;
+  }
+  void release(void* q) {  // hand ownership to the caller
+    for (auto& x : p)
+      if (x == q) x = nullptr;
+  }
+};
+
+int grid_for(uint64_t n) {
+  uint64_t b = (n + 255) / 256;
+  if (b < 1) b = 1;
+  if (b > 148 * 32) b = 148 * 32;
+  return (int)b;
+}
+
+cudaError_t radix_sort(Tmp& t, unsigned long long* in, unsigned long long* out, uint64_t n, int end_bit,
+                       cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  size_t bytes = 0;
+  cudaError_t e = cub::DeviceRadixSort::SortKeys(nullptr, bytes, in, out, (int)n, 0, end_bit, s);
+  if (e != cudaSuccess) return e;
+  void* tmp;
+  e = t.alloc((char**)&tmp, bytes);
+  if (e != cudaSuccess) return e;
+  return cub::DeviceRadixSort::SortKeys(tmp, bytes, in, out, (int)n, 0, end_bit, s);
+}
+
+cudaError_t excl_scan(Tmp& t, const uint32_t* in, uint32_t* out, uint64_t n, cudaStream_t s) {
+  size_t bytes = 0;
+  cudaError_t e = cub::DeviceScan::ExclusiveSum(nullptr, bytes, in, out, (int)n, s);
+  if (e != cudaSuccess) return e;
+  void* tmp;
+  e = t.alloc((char**)&tmp, bytes);
+  if (e != cudaSuccess) return e;
+  return cub::DeviceScan::ExclusiveSum(tmp, bytes, in, out, (int)n, s);
+}
+
+int bits_for(uint64_t x) {
+  int b = 1;
+  while (b < 64 && (1ull << b) <= x) b++;
+  return b;
+}
+
+}  // namespace
+
+extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* edges_uv,
+                                   uint64_t n_edges, const gmbe_load_opts* opts, gmbe_graph** out) {
+  if (!out) return gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: out is NULL");
+  *out = nullptr;
+  if (n_edges && !edges_uv) return gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: edges is NULL");
+  if (n_edges >= (1ull << 32) || n_u >= (1u << 31) || n_v >= (1u << 31))
+    return gmbe_set_error(GMBE_EUNSUPPORTED, "gmbe_load_bipartite: n_edges >= 2^32 or |U|,|V| >= 2^31");
+  gmbe_load_opts o{};
+  o.device = -1;
+  if (opts) {
+    if (opts->struct_size && opts->struct_size < sizeof(uint32_t) * 2)
+      return gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: bad struct_size");
+    o = *opts;
+  }
+  if (o.order > 1) return gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: bad order");
+  int dev = o.device;
+  if (dev < 0) GMBE_CUDA_TRY(cudaGetDevice(&dev));
+  GMBE_CUDA_TRY(cudaSetDevice(dev));
+  cudaStream_t s = (cudaStream_t)o.cuda_stream;
+  bool own = false;
+  if (!s) {
+    GMBE_CUDA_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    own = true;
+  }
+  gmbe_graph* G = new gmbe_graph();
+  G->device = dev;
+  G->stream = s;
+  G->own_stream = own;
+  G->caller_n_u = n_u;
+  G->caller_n_v = n_v;
+  G->order = o.order;
+  G->nbufs = 0;
+  auto fail = [&](int rc) {
+    if (own) cudaStreamDestroy(s);
+    for (int i = 0; i < G->nbufs; i++) cudaFree(G->bufs[i]);
+    delete G;
+    return rc;
+  };
+#define TRY(expr)                                                                           \
+  do {                                                                                      \
+    cudaError_t _e = (expr);                                                                \
+    if (_e != cudaSuccess)                                                                  \
+      return fail(gmbe_set_error(_e == cudaErrorMemoryAllocation ? GMBE_ENOMEM : GMBE_ECUDA, \
+                                 std::string(#expr) + ": " + cudaGetErrorString(_e)));     \
+  } while (0)
+
+  const uint32_t swapped = n_u < n_v ? 1u : 0u;
+  const uint32_t NU = swapped ? n_v : n_u, NV = swapped ? n_u : n_v;
+  const uint64_t m0 = n_edges;
+  Tmp t;
+  // a1: ingest
+  const uint32_t* d_e = edges_uv;
+  if (m0 && !o.edges_on_device) {
+    uint32_t* tmp;
+    TRY(t.alloc(&tmp, 2 * m0));
+    TRY(cudaMemcpyAsync(tmp, edges_uv, 2 * m0 * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
+    d_e = tmp;
+  }
+  unsigned long long *keys, *keys2;
+  int* d_bad;
+  TRY(t.alloc(&keys, m0));
+  TRY(t.alloc(&keys2, m0));
+  TRY(t.alloc(&d_bad, 1));
+  TRY(cudaMemsetAsync(d_bad, 0, sizeof(int), s));
+  if (m0) k_pack_edges<<<grid_for(m0), 256, 0, s>>>(d_e, m0, n_u, n_v, swapped, keys, d_bad);
+  TRY(cudaGetLastError());
+  int h_bad = 0;
+  TRY(cudaMemcpyAsync(&h_bad, d_bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+  TRY(cudaStreamSynchronize(s));
+  if (h_bad) return fail(gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: edge id out of range"));
+  TRY(radix_sort(t, keys, keys2, m0, 32 + bits_for(NU), s));
+  // unique
+  uint64_t m = 0;
+  if (m0) {
+    int* d_num;
+    TRY(t.alloc(&d_num, 1));
+    size_t bytes = 0;
+    TRY(cub::DeviceSelect::Unique(nullptr, bytes, keys2, keys, d_num, (int)m0, s));
+    char* tmp;
+    TRY(t.alloc(&tmp, bytes));
+    TRY(cub::DeviceSelect::Unique(tmp, bytes, keys2, keys, d_num, (int)m0, s));
+    int hn = 0;
+    TRY(cudaMemcpyAsync(&hn, d_num, sizeof(int), cudaMemcpyDeviceToHost, s));
+    TRY(cudaStreamSynchronize(s));
+    m = (uint64_t)hn;
+  }
+  // a2: degrees and order
+  uint32_t *deg_u, *deg_v, *deg_by_rank, *id2rank, *maxes;
+  TRY(t.alloc(&deg_u, NU + 1));
+  TRY(t.alloc(&deg_v, NV + 1));
+  TRY(t.alloc(&deg_by_rank, NV + 1));
+  TRY(t.alloc(&id2rank, NV + 1));
+  TRY(t.alloc(&maxes, 4));
+  TRY(cudaMemsetAsync(deg_u, 0, (NU + 1) * sizeof(uint32_t), s));
+  TRY(cudaMemsetAsync(deg_v, 0, (NV + 1) * sizeof(uint32_t), s));
+  TRY(cudaMemsetAsync(deg_by_rank, 0, (NV + 1) * sizeof(uint32_t), s));
+  TRY(cudaMemsetAsync(maxes, 0, 4 * sizeof(uint32_t), s));
+  if (m) k_degrees<<<grid_for(m), 256, 0, s>>>(keys, m, deg_u, deg_v);
+  unsigned long long *okeys, *okeys2;
+  TRY(t.alloc(&okeys, NV));
+  TRY(t.alloc(&okeys2, NV));
+  if (NV) k_order_keys<<<grid_for(NV), 256, 0, s>>>(deg_v, NV, o.order == GMBE_ORDER_IDENTITY, okeys);
+  TRY(radix_sort(t, okeys, okeys2, NV, 32 + bits_for(m + 1), s));
+  // persistent buffers
+  uint32_t *off_v, *adj_v, *off_u, *adj_u, *rank2id;
+  unsigned long long* hv;
+  TRY(t.alloc(&off_v, NV + 1));
+  TRY(t.alloc(&adj_v, m));
+  TRY(t.alloc(&off_u, NU + 1));
+  TRY(t.alloc(&adj_u, m));
+  TRY(t.alloc(&rank2id, NV));
+  TRY(t.alloc(&hv, NV));
+  // library V side == caller V (hash side 1) unless swapped (then caller U, side 0)
+  if (NV)
+    k_rank_maps<<<grid_for(NV), 256, 0, s>>>(okeys2, NV, swapped ? 0u : 1u, rank2id, id2rank, deg_v,
+                                             deg_by_rank, hv);
+  TRY(excl_scan(t, deg_by_rank, off_v, (uint64_t)NV + 1, s));
+  TRY(excl_scan(t, deg_u, off_u, (uint64_t)NU + 1, s));
+  if (m) {
+    unsigned long long *kv, *ku;
+    TRY(t.alloc(&kv, m));
+    TRY(t.alloc(&ku, m));
+    k_rekey<<<grid_for(m), 256, 0, s>>>(keys, m, id2rank, kv, ku);
+    TRY(radix_sort(t, kv, keys2, m, 32 + bits_for(NV), s));
+    k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_v);
+    TRY(radix_sort(t, ku, keys2, m, 32 + bits_for(NU), s));
+    k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_u);
+  }
+  if (NV || NU) k_bounds<<<grid_for((uint64_t)NV * 32 + NU), 256, 0, s>>>(off_v, adj_v, off_u, NV, NU, maxes);
+  TRY(cudaGetLastError());
+  uint32_t hm[4];
+  TRY(cudaMemcpyAsync(hm, maxes, sizeof(hm), cudaMemcpyDeviceToHost, s));
+  TRY(cudaStreamSynchronize(s));
+
+  void* keep[] = {off_v, adj_v, off_u, adj_u, rank2id, hv};
+  for (void* q : keep) {
+    t.release(q);
+    G->bufs[G->nbufs++] = q;
+  }
+  DevGraph& g = G->g;
+  g.n_u = NU;
+  g.n_v = NV;
+  g.m = m;
+  g.swapped = swapped;
+  g.off_v = off_v;
+  g.adj_v = adj_v;
+  g.off_u = off_u;
+  g.adj_u = adj_u;
+  g.rank2id = rank2id;
+  g.hv = hv;
+  g.delta_v = hm[0];
+  g.delta_u = hm[1];
+  g.wedge_bound = hm[2];
+  *out = G;
+  return GMBE_OK;
+#undef TRY
+}
+
+extern "C" int gmbe_graph_info_get(const gmbe_graph* G, gmbe_graph_info* out) {
+  if (!G || !out) return gmbe_set_error(GMBE_EINVAL, "gmbe_graph_info_get: NULL argument");
+  out->n_u = G->caller_n_u;
+  out->n_v = G->caller_n_v;
+  out->n_edges_unique = G->g.m;
+  out->delta_u = G->g.delta_u;
+  out->delta_v = G->g.delta_v;
+  // Σ_{u∈N(v)} (|N(u)| - 1) = wedges - |N(v)|; bounded by the max wedge count
+  out->wedge_bound_v = G->g.wedge_bound;
+  out->swapped = G->g.swapped;
+  out->order = G->order;
+  out->device = (uint32_t)G->device;
+  return GMBE_OK;
+}
+
+extern "C" void gmbe_free_graph(gmbe_graph* G) {
+  if (!G) return;
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(G->device);
+  cudaStreamSynchronize(G->stream);
+  gmbe_release_workspace(G);
+  for (int i = 0; i < G->nbufs; i++) cudaFree(G->bufs[i]);
+  if (G->own_stream) cudaStreamDestroy(G->stream);
+  cudaSetDevice(prev);
+  delete G;
+}

@@ -1,0 +1,245 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by element.
+
+Count and checksum must be bit-exact; on small inputs the full biclique SET must be equal; the
+canonical-tree counters (nodes, nonmax, algo_bytes) must match exactly (schedule-independent,
+DESIGN.md reading A9).  Marked gpu: run on the B200 box."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from gmbe_inputs import complete_edges, crown_edges, g0_edges, make_config, matching_edges, star_edges
+
+pytestmark = pytest.mark.gpu
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+@pytest.fixture(scope="module")
+def gmbe():
+    import torch
+    assert torch.cuda.is_available()
+    import paper_conf_sc_panhlzwc23_b200 as m
+    return m
+
+
+def _run(gmbe, nu, nv, e, order="degree", **kw):
+    g = gmbe.load(nu, nv, e, order=order)
+    try:
+        return g.enumerate(**kw)
+    finally:
+        g.free()
+
+
+def _same(r, o, counters=True):
+    assert (r.count, r.checksum) == (o.count, o.checksum)
+    if counters:
+        assert (r.roots_run, r.nodes, r.nonmax) == (o.roots_run, o.nodes, o.nonmax)
+
+
+# ---------------------------------------------------------------- paper worked example
+def test_g0_sets_and_tree(gmbe):
+    nu, nv, e = g0_edges()
+    for order in ("identity", "degree"):
+        for prune in (True, False):
+            r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True, counters=True,
+                     per_root=True)
+            o = oracle.oracle_mbe(nu, nv, e, order=order, prune=prune, records=True, per_root=True)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques)
+            assert (r.algo_bytes, r.algo_bytes_qfull) == (o.algo_bytes, o.algo_bytes_qfull)
+            assert r.per_root_count.tolist() == o.per_root_count.tolist()
+    # Fig 2 / Ex 4.1: identity order, t1 pruned
+    r = _run(gmbe, nu, nv, e, order="identity")
+    assert (r.count, r.nodes, r.nonmax, r.roots_run) == (6, 3, 0, 3)
+
+
+# ---------------------------------------------------------------- random tiny graphs
+def _rand_graph(rng, nmax=10):
+    nu = int(rng.integers(1, nmax))
+    nv = int(rng.integers(1, nmax))
+    p = float(rng.choice([0.2, 0.35, 0.5, 0.65, 0.8]))
+    e = np.argwhere(rng.random((nu, nv)) < p).astype(np.uint32)
+    if len(e) and rng.random() < 0.3:
+        e = np.concatenate([e, e[rng.integers(0, len(e), size=3)]])
+    return nu, nv, e
+
+
+def test_random_tiny_sets(gmbe):
+    rng = np.random.default_rng(99)
+    for _ in range(300):
+        nu, nv, e = _rand_graph(rng)
+        order = "degree" if rng.random() < 0.7 else "identity"
+        prune = bool(rng.random() < 0.8)
+        r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True, counters=True)
+        o = oracle.oracle_mbe(nu, nv, e, order=order, prune=prune, records=True)
+        _same(r, o)
+        assert r.bicliques == sorted(o.bicliques)
+        assert r.algo_bytes == o.algo_bytes
+
+
+def test_random_medium_dense(gmbe):
+    """Denser and larger than tiny: spans several 32-bit words per row (W > 1) and ragged tails."""
+    rng = np.random.default_rng(5)
+    for it in range(40):
+        nu = int(rng.integers(20, 140))
+        nv = int(rng.integers(10, 60))
+        p = float(rng.uniform(0.05, 0.35))
+        e = np.argwhere(rng.random((nu, nv)) < p).astype(np.uint32)
+        r = _run(gmbe, nu, nv, e, counters=True)
+        o = oracle.oracle_mbe(nu, nv, e)
+        _same(r, o)
+        assert (r.algo_bytes, r.algo_bytes_qfull) == (o.algo_bytes, o.algo_bytes_qfull)
+
+
+# ---------------------------------------------------------------- closed forms / edge cases
+def test_closed_forms(gmbe):
+    for n in range(2, 15):
+        nu, nv, e = crown_edges(n)
+        r = _run(gmbe, nu, nv, e)
+        assert r.count == 2 ** n - 2
+        if n <= 10:
+            o = oracle.oracle_mbe(nu, nv, e)
+            _same(r, o)
+    for a, b in ((1, 1), (3, 5), (40, 2), (33, 70)):
+        r = _run(gmbe, *complete_edges(a, b), records=True)
+        assert r.count == 1 and r.bicliques == [(tuple(range(a)), tuple(range(b)))]
+    r = _run(gmbe, *matching_edges(50))
+    assert r.count == 50
+    r = _run(gmbe, *star_edges(100))
+    assert r.count == 1
+    r = _run(gmbe, 7, 9, np.zeros((0, 2), np.uint32))
+    assert (r.count, r.checksum) == (0, 0)
+
+
+def test_invalid_ids(gmbe):
+    with pytest.raises(gmbe.GmbeError) as ei:
+        gmbe.load(3, 3, np.array([[0, 3]], np.uint32))
+    assert ei.value.code == gmbe.GMBE_EINVAL
+
+
+def test_swapped_orientation_sets(gmbe):
+    """|U| < |V|: the library swaps sides internally; output stays in caller roles."""
+    rng = np.random.default_rng(12)
+    for _ in range(50):
+        nu = int(rng.integers(1, 8))
+        nv = int(rng.integers(nu + 1, 14))
+        e = np.argwhere(rng.random((nu, nv)) < 0.45).astype(np.uint32)
+        r = _run(gmbe, nu, nv, e, records=True)
+        o = oracle.oracle_mbe(nu, nv, e, records=True)
+        _same(r, o)
+        assert r.bicliques == sorted(o.bicliques)
+
+
+# ---------------------------------------------------------------- ER(40,40,.15)
+def test_er40(gmbe):
+    nu, nv, e = make_config("er40")
+    for prune in (True, False):
+        r = _run(gmbe, nu, nv, e, prune=prune, records=True, counters=True)
+        o = oracle.oracle_mbe(nu, nv, e, prune=prune, records=True)
+        _same(r, o)
+        assert r.count == 211
+        assert r.bicliques == sorted(o.bicliques)
+        assert (r.algo_bytes, r.algo_bytes_qfull) == (o.algo_bytes, o.algo_bytes_qfull)
+
+
+# ---------------------------------------------------------------- schedule freedom (A9)
+@pytest.fixture(scope="module")
+def dense_case():
+    rng = np.random.default_rng(2024)
+    nu, nv = 90, 60
+    a = rng.random((nu, nv)) < 0.12
+    a[:24, :20] |= rng.random((24, 20)) < 0.75  # one dense block -> deep, heavy subtrees
+    e = np.argwhere(a).astype(np.uint32)
+    o = oracle.oracle_mbe(nu, nv, e, records=True)
+    return nu, nv, e, o
+
+
+def test_split_and_schedule_invariance(gmbe, dense_case):
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        variants = [dict(), dict(split=False), dict(bound_height=1, bound_size=1),
+                    dict(bound_height=1, bound_size=1, n_slabs=1),
+                    dict(bound_height=1, bound_size=1, n_slabs=3, slab_words=4096),
+                    dict(warps_per_sm=8), dict(warps_per_sm=64)]
+        for kw in variants:
+            r = g.enumerate(counters=True, **kw)
+            _same(r, o)
+            assert r.algo_bytes == o.algo_bytes, kw
+        r = g.enumerate(bound_height=1, bound_size=1, records=True)
+        assert r.tasks > 0 and r.splits > 0
+        assert r.bicliques == sorted(o.bicliques)
+    finally:
+        g.free()
+
+
+def test_parts_are_additive(gmbe, dense_case):
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        for n in (2, 3, 8):
+            rs = [g.enumerate(part=(i, n), counters=True) for i in range(n)]
+            assert sum(x.count for x in rs) == o.count
+            assert sum(x.checksum for x in rs) % (1 << 64) == o.checksum
+            assert sum(x.nodes for x in rs) == o.nodes
+            assert sum(x.algo_bytes for x in rs) == o.algo_bytes
+            for i in range(n):  # per-shard parity (ownership invariant)
+                os_ = oracle.oracle_mbe(nu, nv, e, shard=(i, n))
+                assert (rs[i].count, rs[i].checksum) == (os_.count, os_.checksum)
+    finally:
+        g.free()
+
+
+def test_output_truncation(gmbe, dense_case):
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        r = g.enumerate(records=True, rec_cap=10, ids_cap=1 << 20)
+        assert r.truncated == 1 and r.count == o.count and r.checksum == o.checksum
+        assert r.n_written == 10 and set(r.bicliques) <= set(o.bicliques)
+        r = g.enumerate(records=True, rec_cap=1 << 16, ids_cap=100)
+        assert r.truncated == 1 and r.count == o.count
+    finally:
+        g.free()
+
+
+def test_device_edges_and_duplicates(gmbe):
+    import torch
+    nu, nv, e = make_config("er40")
+    dup = np.concatenate([e, e[::3]])
+    t = torch.from_numpy(dup.astype(np.int32)).cuda()
+    g = gmbe.load(nu, nv, t)
+    r = g.enumerate()
+    info = g.info()
+    g.free()
+    assert info["n_edges_unique"] == 239
+    assert (r.count, r.checksum) == (211, 0x357D6B7B401275D4)
+
+
+# ---------------------------------------------------------------- full-size configs
+def _gold_cfg():
+    p = os.path.join(GOLD, "configs_oracle.json")
+    with open(p) as f:
+        return json.load(f)
+
+
+@pytest.mark.parametrize("name", ["yg", "gh", "dblp", "bx", "gh_work"])
+def test_full_config_vs_oracle_golden(gmbe, name):
+    gold = _gold_cfg()
+    if name not in gold:
+        pytest.skip("no golden for %s" % name)
+    gd = gold[name]
+    nu, nv, e = make_config(name)
+    g = gmbe.load(nu, nv, e)
+    try:
+        r = g.enumerate(counters=True)
+        assert (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16))
+        assert (r.nodes, r.nonmax, r.roots_run) == (gd["nodes"], gd["nonmax"], gd["roots_run"])
+        assert (r.algo_bytes, r.algo_bytes_qfull) == (gd["algo_bytes"], gd["algo_bytes_qfull"])
+        r2 = g.enumerate()  # the bench launch configuration (no counters)
+        assert (r2.count, r2.checksum) == (r.count, r.checksum)
+    finally:
+        g.free()
