@@ -1,0 +1,303 @@
+"""bench.py -- maximal bicliques/sec on a Github-shaped synthetic bipartite graph, 1..8 B200.
+
+One STEP = one pass of the whole hot path (DESIGN.md a1-a8) over the workload: device graph build
+from device-resident edges (gmbe_load_bipartite) + enumeration (gmbe_enumerate) of this rank's
+root shard + (N > 1) the NCCL all-reduce of [count, checksum, ...].  `value` = bicliques of the
+whole graph / max-over-ranks step time.  `e2e` repeats the step through the public API with the
+edges in pinned HOST memory (H2D inside the timed region) and the result read back to the host.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config gh_work] [--impl reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+DEFAULT_CONFIG = "gh_work"
+METRIC = "maximal bicliques/sec (Github-shaped)"
+CTRL_D2H_BYTES = 144  # sizeof(Ctrl) read back by gmbe_enumerate (gmbe_enum.cu)
+
+
+def _args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default=DEFAULT_CONFIG)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget-s", type=float, default=15.0)
+    return ap.parse_args()
+
+
+def _dist():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def _gold(name):
+    p = os.path.join(ROOT, "tests", "golden", "configs_oracle.json")
+    try:
+        with open(p) as f:
+            return json.load(f).get(name)
+    except OSError:
+        return None
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def _traffic(name):
+    """DRAM bytes per k_enum launch from the committed ncu --set full summary, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d[name]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
+def _cpu_sample(name, budget_s, gold):
+    """Time the oracle (as it stands, 1 thread) on a bounded root shard of the workload."""
+    import oracle
+    from gmbe_inputs import make_config
+    nu, nv, e = make_config(name)
+    if gold and gold.get("oracle_cpu_seconds"):
+        shards = max(1, int(round(gold["oracle_cpu_seconds"] / budget_s)))
+    else:
+        shards = 256
+        while True:
+            t = time.time()
+            oracle.oracle_mbe(nu, nv, e, shard=(0, shards))
+            dt = time.time() - t
+            if dt * 8 > budget_s or shards == 1:
+                shards = max(1, int(shards * dt / budget_s)) if dt > 0 else shards
+                break
+            shards //= 8
+    t = time.time()
+    r = oracle.oracle_mbe(nu, nv, e, shard=(0, shards))
+    dt = time.time() - t
+    return r, dt, shards
+
+
+class ClockSampler:
+    def __init__(self, index):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(index), "--query-gpu=" + q,
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        self.p.wait()
+        self.f.seek(0)
+        rows = [r.split(",") for r in self.f.read().strip().splitlines() if r.strip()]
+        os.unlink(self.f.name)
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[1]))
+                mx = max(mx, float(r[2]))
+                for n, v in zip(names, r[5:9]):
+                    if v.strip() == "Active":
+                        reasons.add(n)
+            except (ValueError, IndexError):
+                pass
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def run_reference(a):
+    """Reference arm: the CPU oracle as it stands, on the host cores, same metric and workload."""
+    ws, rank, _ = _dist()
+    if rank != 0:
+        return
+    from gmbe_inputs import make_config
+    gold = _gold(a.config)
+    nu, nv, e = make_config(a.config)
+    for _ in range(max(0, min(a.warmup, 1))):
+        _cpu_sample(a.config, a.cpu_budget_s / 4, gold)
+    times, counts, shards = [], [], 1
+    for _ in range(a.steps):
+        r, dt, shards = _cpu_sample(a.config, a.cpu_budget_s, gold)
+        times.append(dt)
+        counts.append(r.count)
+    v = sum(counts) / sum(times)
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "bicliques/s",
+            "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup,
+            "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": a.config, "n_u": nu, "n_v": nv, "m": int(len(e)),
+                       "sample": "root shard 0/%d" % shards},
+            "cpu_baseline": {"value": v, "unit": "bicliques/s", "cores": 1, "kind": "oracle",
+                             "sample": "oracle single-thread on root shard 0/%d of %s" % (shards, a.config)},
+            "e2e": {"value": v, "unit": "bicliques/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    a = _args()
+    if a.impl == "reference":
+        return run_reference(a)
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_panhlzwc23_b200 as gmbe
+    from gmbe_inputs import make_config, graph_stats
+
+    ws, rank, local = _dist()
+    assert ws == a.gpus or ws == 1, "launch with torchrun --nproc-per-node %d" % a.gpus
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    nu, nv, e = make_config(a.config)
+    m = len(e)
+    e_dev = torch.from_numpy(e.astype(np.int32)).to(dev)                   # resident in HBM
+    e_host = torch.from_numpy(e.astype(np.int32)).pin_memory()             # for the e2e leg
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)          # > 126 MB L2
+    part = (rank, ws)
+
+    def step(edges, kernel_ms):
+        g = gmbe.load(nu, nv, edges, device=local, stream=stream)
+        r = g.enumerate(part=part, stream=stream)
+        g.free()
+        kernel_ms.append(r.kernel_ms)
+        res = torch.tensor([r.count, r.checksum - (1 << 64) if r.checksum >= 1 << 63 else r.checksum,
+                            r.nodes, r.nonmax], dtype=torch.int64, device=dev)
+        if ws > 1:
+            dist.all_reduce(res)  # the only cross-GPU exchange (NVLink / NVSwitch)
+        return res
+
+    # canonical work of this shard (counters run, untimed; identical in every schedule)
+    g = gmbe.load(nu, nv, e_dev, device=local, stream=stream)
+    info = g.info()
+    rc = g.enumerate(part=part, counters=True, stream=stream)
+    g.free()
+
+    kms = []
+    for _ in range(a.warmup):
+        step(e_dev, kms)
+    torch.cuda.synchronize(dev)
+    if ws > 1:
+        dist.barrier()
+    launches0 = gmbe.kernel_launch_count()
+    clk = ClockSampler(local)
+    kms = []
+    dev_ms = []
+    res = None
+    for _ in range(a.steps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        res = step(e_dev, kms)
+        e1.record(stream)
+        e1.synchronize()
+        dev_ms.append(e0.elapsed_time(e1))
+    torch.cuda.synchronize(dev)
+    clocks = clk.stop()
+    launches = gmbe.kernel_launch_count() - launches0
+    # e2e: edges from pinned host memory, result back on the host, per step
+    e2e_ms = []
+    for _ in range(a.steps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        g = gmbe.load(nu, nv, e_host.numpy(), device=local, stream=stream)
+        r = g.enumerate(part=part, stream=stream)
+        g.free()
+        rr = torch.tensor([r.count], dtype=torch.int64, device=dev)
+        if ws > 1:
+            dist.all_reduce(rr)
+        total_e2e = int(rr.item())
+        e1.record(stream)
+        e1.synchronize()
+        e2e_ms.append(e0.elapsed_time(e1))
+
+    t_rank = sum(dev_ms) / len(dev_ms)
+    t_e2e = sum(e2e_ms) / len(e2e_ms)
+    k_rank = sum(kms) / len(kms)
+    tt = torch.tensor([t_rank, t_e2e], dtype=torch.float64, device=dev)
+    if ws > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    t_step, t_e2e = float(tt[0]), float(tt[1])
+    count = int(res[0].item())
+    checksum = int(res[1].item()) % (1 << 64)
+    assert total_e2e == count
+
+    if rank == 0:
+        gold = _gold(a.config)
+        parity = None
+        if gold:
+            parity = (count == gold["count"] and checksum == int(gold["checksum"], 16))
+        peak, peak_kind = _peaks()
+        achieved = rc.algo_bytes / (k_rank * 1e-3) / 1e9 if k_rank > 0 else 0.0
+        st = graph_stats(nu, nv, e)
+        line = {
+            "metric": METRIC, "value": count / (t_step * 1e-3), "unit": "bicliques/s",
+            "n_gpus": ws, "steps": a.steps, "warmup": a.warmup, "ms_per_step": t_step,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "u32", "data": "synthetic",
+            "config": {"workload": a.config, "n_u": nu, "n_v": nv, "m": st["m"],
+                       "delta_u": st["delta_u"], "delta_v": st["delta_v"], "seed": 0,
+                       "bicliques": count, "checksum": hex(checksum), "oracle_parity": parity,
+                       "parallelism": "root-shard x%d (degree-rank interleave) + NCCL all-reduce" % ws,
+                       "l2": "flushed between steps (256 MiB memset)",
+                       "step": "device CSR build + enumerate (+ all-reduce)"},
+            "kernel_ms": k_rank,
+            "e2e": {"value": count / (t_e2e * 1e-3), "unit": "bicliques/s",
+                    "h2d_bytes_per_step": int(m * 8), "d2h_bytes_per_step": CTRL_D2H_BYTES},
+            "gpu_launches": int(launches),
+            "roofline": {"bound": "hbm", "kernel": "k_enum", "achieved": achieved, "peak": peak,
+                         "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak,
+                         "traffic": _traffic(a.config),
+                         "algo_bytes_per_launch": rc.algo_bytes, "algo_bytes_qfull": rc.algo_bytes_qfull},
+            "work": {"nodes": rc.nodes, "nonmax": rc.nonmax, "roots_run": rc.roots_run,
+                     "splits": rc.splits, "tasks": rc.tasks},
+            "clocks": clocks,
+        }
+        if ws == 1 and not a.no_cpu_baseline:
+            r, dt, shards = _cpu_sample(a.config, a.cpu_budget_s, gold)
+            line["cpu_baseline"] = {"value": r.count / dt, "unit": "bicliques/s", "cores": 1,
+                                    "kind": "oracle",
+                                    "sample": "root shard 0/%d (%d bicliques, %.1f s)" % (shards, r.count, dt)}
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -136,9 +136,14 @@ typedef struct {
  * Errors: EINVAL (NULL g/out, part_index >= part_count), ENOMEM, ECUDA, EINTERNAL. */
 int gmbe_enumerate(const gmbe_graph* g, const gmbe_opts* opts, gmbe_result* out);
 
-/* Free the device workspace (node-stack arenas, task slabs) cached on g by gmbe_enumerate.
- * Optional: gmbe_free_graph releases it too.  NULL-safe. */
+/* gmbe_enumerate keeps its device workspace (node-stack arenas, task slabs, queues) in a
+ * per-device pool for reuse by later calls.  This frees the idle workspaces of g's device.
+ * NULL-safe. */
 void gmbe_release_workspace(const gmbe_graph* g);
+
+/* Number of this library's own kernels launched so far in this process (all devices); CUB
+ * primitives used by the graph build are not counted. */
+uint64_t gmbe_kernel_launch_count(void);
 
 const char* gmbe_last_error(void);
 

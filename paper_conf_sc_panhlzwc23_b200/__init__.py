@@ -24,6 +24,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 GMBE_OK, GMBE_EINVAL, GMBE_ENOMEM, GMBE_ECUDA, GMBE_EUNSUPPORTED, GMBE_EINTERNAL = 0, -1, -2, -3, -4, -5
 ORDER = {"degree": 0, "identity": 1}
 EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmbe_node_buf_bound_bytes",
+           "gmbe_kernel_launch_count",
            "gmbe_naive_alloc_bytes", "gmbe_enumerate", "gmbe_release_workspace", "gmbe_last_error")
 
 _u32, _i32, _u64, _vp = ctypes.c_uint32, ctypes.c_int32, ctypes.c_uint64, ctypes.c_void_p
@@ -69,6 +70,8 @@ _lib.gmbe_naive_alloc_bytes.argtypes = [_u64, _u64]
 _lib.gmbe_naive_alloc_bytes.restype = _u64
 _lib.gmbe_enumerate.argtypes = [_vp, ctypes.POINTER(Opts), ctypes.POINTER(CResult)]
 _lib.gmbe_enumerate.restype = ctypes.c_int
+_lib.gmbe_kernel_launch_count.argtypes = []
+_lib.gmbe_kernel_launch_count.restype = _u64
 _lib.gmbe_last_error.argtypes = []
 _lib.gmbe_last_error.restype = ctypes.c_char_p
 
@@ -82,6 +85,11 @@ class GmbeError(RuntimeError):
 def _check(rc):
     if rc != GMBE_OK:
         raise GmbeError(rc, _lib.gmbe_last_error().decode(errors="replace"))
+
+
+def kernel_launch_count():
+    """Number of libgmbe kernels launched so far in this process."""
+    return int(_lib.gmbe_kernel_launch_count())
 
 
 def node_buf_bound_bytes(delta_v, delta2_v):

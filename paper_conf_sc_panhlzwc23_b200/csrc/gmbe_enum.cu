@@ -469,7 +469,8 @@ __device__ uint32_t slab_alloc(const Params& P) {
 __device__ void slab_free(const Params& P, uint32_t s) {
   if (lane_id() == 0) ring_push(P.fq, P.ring_mask, &P.ctrl->f_tail, s);
 }
-// slab layout: [0]=W [1]=map length [2]=root rank [3]=R length [4..7] pad | map | R list | node
+// slab layout: [0]=W [1]=map length [2]=root rank [3]=R length [4]=node offset [5..7] pad |
+//              map | R list | node
 __device__ __forceinline__ uint32_t slab_node_off(uint32_t lmap, uint32_t rlen) {
   return kHdr + r4(lmap) + r4(rlen);
 }
@@ -501,9 +502,10 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     const uint64_t need = kHdr + T.W4 + (uint64_t)max_entries * T.E;
     uint32_t slab = kNone;
     uint32_t* ch;
+    uint32_t node_off = 0;
     if (split_mode && cur == top) {
       const uint32_t rlen_max = T.rlist ? cur[5] + 1 + cur[0] : 0;
-      const uint64_t node_off = slab_node_off(lmap, rlen_max);
+      node_off = slab_node_off(lmap, rlen_max);
       if (node_off + need <= P.slab_words) slab = slab_alloc(P);
       if (slab != kNone) ch = P.slabs + (uint64_t)slab * P.slab_words + node_off;
     }
@@ -528,6 +530,7 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
           s[1] = lmap;
           s[2] = T.root;
           s[3] = rlen;
+          s[4] = node_off;
           ch[4] = kNone;
           ch[3] = 0;
         }
@@ -827,7 +830,7 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       if (rbuf)
         for (uint32_t j = lane; j < rlen; j += 32) rbuf[j] = s[kHdr + r4(lmap) + j];
       __syncwarp();
-      uint32_t* top = s + slab_node_off(lmap, rbuf ? rlen : 0);
+      uint32_t* top = s + s[4];
       dispatch_task(P, Tc, top, arena, arena + P.arena_words, lmap, A);
       __syncwarp();
       slab_free(P, task);
@@ -911,15 +914,12 @@ cudaError_t ensure(void** p, size_t* have, size_t need) {
 
 }  // namespace
 
-// Workspace cache, one per graph handle (freed with the graph).
-struct GmbeWs {
-  Workspace w;
-};
 
 extern "C" uint64_t gmbe_node_buf_bound_bytes(uint64_t dv, uint64_t d2v) { return (3 * dv + 2 * d2v) * 4; }
 extern "C" uint64_t gmbe_naive_alloc_bytes(uint64_t dv, uint64_t d2v) { return dv * (dv + d2v) * 4; }
 
-static Workspace* ws_of(const gmbe_graph* G);
+static Workspace* ws_acquire(int device);
+static void ws_return(Workspace* w);
 
 extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_result* out) {
   if (!G || !out) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: NULL argument");
@@ -933,7 +933,12 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   cudaStream_t s = o.cuda_stream ? (cudaStream_t)o.cuda_stream : G->stream;
   const DevGraph& g = G->g;
   std::memset(out, 0, sizeof(*out));
-  Workspace& W = *ws_of(G);
+  Workspace* Wp = ws_acquire(G->device);
+  struct Ret {
+    Workspace* w;
+    ~Ret() { ws_return(w); }
+  } ret{Wp};
+  Workspace& W = *Wp;
 
   int sms = 0;
   GMBE_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, G->device));
@@ -1013,13 +1018,14 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   GMBE_CUDA_TRY(cudaMemcpyAsync(W.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
   k_init_rings<<<(cap + 255) / 256 < 1024 ? (cap + 255) / 256 : 1024, 256, 0, s>>>(P.tq, P.fq, cap,
                                                                                     (uint32_t)n_slabs);
+  gmbe_note_launch();
   if (P.per_root) GMBE_CUDA_TRY(cudaMemsetAsync(W.per_root, 0, (size_t)(g.n_v + 1) * 8, s));
   GMBE_CUDA_TRY(cudaGetLastError());
   cudaEvent_t e0, e1;
   GMBE_CUDA_TRY(cudaEventCreate(&e0));
   GMBE_CUDA_TRY(cudaEventCreate(&e1));
   GMBE_CUDA_TRY(cudaEventRecord(e0, s));
-  if (P.n_roots > 0) k_enum<<<blocks, 256, 0, s>>>(P);
+  if (P.n_roots > 0) k_enum<<<blocks, 256, 0, s>>>(P), gmbe_note_launch();
   cudaError_t le = cudaGetLastError();
   GMBE_CUDA_TRY(cudaEventRecord(e1, s));
   GMBE_CUDA_TRY(le);
@@ -1055,23 +1061,43 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   return GMBE_OK;
 }
 
-#include <map>
 #include <mutex>
+// Workspace pool: a call takes an idle workspace of its device (or a new one) and returns it, so
+// repeated calls reuse device memory and concurrent calls never share one.
 static std::mutex g_ws_mu;
-static std::map<const gmbe_graph*, Workspace*> g_ws;
-static Workspace* ws_of(const gmbe_graph* G) {
+static std::vector<Workspace*> g_ws_idle;
+static Workspace* ws_acquire(int device) {
   std::lock_guard<std::mutex> lk(g_ws_mu);
-  Workspace*& w = g_ws[G];
-  if (!w) w = new Workspace();
+  for (size_t i = 0; i < g_ws_idle.size(); i++)
+    if (g_ws_idle[i]->device == device) {
+      Workspace* w = g_ws_idle[i];
+      g_ws_idle.erase(g_ws_idle.begin() + i);
+      return w;
+    }
+  Workspace* w = new Workspace();
+  w->device = device;
   return w;
 }
-extern "C" void gmbe_release_workspace(const gmbe_graph* G) {
+static void ws_return(Workspace* w) {
   std::lock_guard<std::mutex> lk(g_ws_mu);
-  auto it = g_ws.find(G);
-  if (it == g_ws.end()) return;
-  Workspace* w = it->second;
-  for (void* p : {w->arena, w->slabs, w->rings, w->rbuf, w->ctrl, w->per_root})
-    if (p) cudaFree(p);
-  delete w;
-  g_ws.erase(it);
+  g_ws_idle.push_back(w);
+}
+extern "C" void gmbe_release_workspace(const gmbe_graph* G) {
+  if (!G) return;
+  std::lock_guard<std::mutex> lk(g_ws_mu);
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(G->device);
+  for (size_t i = 0; i < g_ws_idle.size();) {
+    Workspace* w = g_ws_idle[i];
+    if (w->device != G->device) {
+      i++;
+      continue;
+    }
+    for (void* p : {w->arena, w->slabs, w->rings, w->rbuf, w->ctrl, w->per_root})
+      if (p) cudaFree(p);
+    delete w;
+    g_ws_idle.erase(g_ws_idle.begin() + i);
+  }
+  cudaSetDevice(prev);
 }

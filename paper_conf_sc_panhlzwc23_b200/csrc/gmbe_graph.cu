@@ -106,15 +106,19 @@ __global__ void k_bounds(const uint32_t* __restrict__ off_v, const uint32_t* __r
     atomicMax(&maxes[1], off_u[u + 1] - off_u[u]);
 }
 
+// stream-ordered allocations from the device's default pool (cheap to repeat per step)
 struct Tmp {
+  cudaStream_t s;
   std::vector<void*> p;
+  explicit Tmp(cudaStream_t st) : s(st) {}
   ~Tmp() {
-    for (void* x : p) cudaFree(x);
+    for (void* x : p)
+      if (x) cudaFreeAsync(x, s);
   }
   template <class T>
   cudaError_t alloc(T** out, size_t n) {
     void* q = nullptr;
-    cudaError_t e = cudaMalloc(&q, n ? n * sizeof(T) : 16);
+    cudaError_t e = cudaMallocAsync(&q, n ? n * sizeof(T) : 16, s);
     if (e == cudaSuccess) p.push_back(q);
     *out = (T*)q;
     return e;
@@ -186,6 +190,14 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
     GMBE_CUDA_TRY(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
     own = true;
   }
+  {
+    // keep freed pool memory cached across calls instead of returning it at every sync
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = ~0ull;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
   gmbe_graph* G = new gmbe_graph();
   G->device = dev;
   G->stream = s;
@@ -195,8 +207,9 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   G->order = o.order;
   G->nbufs = 0;
   auto fail = [&](int rc) {
+    for (int i = 0; i < G->nbufs; i++) cudaFreeAsync(G->bufs[i], s);
+    cudaStreamSynchronize(s);
     if (own) cudaStreamDestroy(s);
-    for (int i = 0; i < G->nbufs; i++) cudaFree(G->bufs[i]);
     delete G;
     return rc;
   };
@@ -211,7 +224,7 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   const uint32_t swapped = n_u < n_v ? 1u : 0u;
   const uint32_t NU = swapped ? n_v : n_u, NV = swapped ? n_u : n_v;
   const uint64_t m0 = n_edges;
-  Tmp t;
+  Tmp t(s);
   // a1: ingest
   const uint32_t* d_e = edges_uv;
   if (m0 && !o.edges_on_device) {
@@ -226,7 +239,7 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   TRY(t.alloc(&keys2, m0));
   TRY(t.alloc(&d_bad, 1));
   TRY(cudaMemsetAsync(d_bad, 0, sizeof(int), s));
-  if (m0) k_pack_edges<<<grid_for(m0), 256, 0, s>>>(d_e, m0, n_u, n_v, swapped, keys, d_bad);
+  if (m0) k_pack_edges<<<grid_for(m0), 256, 0, s>>>(d_e, m0, n_u, n_v, swapped, keys, d_bad), gmbe_note_launch();
   TRY(cudaGetLastError());
   int h_bad = 0;
   TRY(cudaMemcpyAsync(&h_bad, d_bad, sizeof(int), cudaMemcpyDeviceToHost, s));
@@ -259,11 +272,11 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   TRY(cudaMemsetAsync(deg_v, 0, (NV + 1) * sizeof(uint32_t), s));
   TRY(cudaMemsetAsync(deg_by_rank, 0, (NV + 1) * sizeof(uint32_t), s));
   TRY(cudaMemsetAsync(maxes, 0, 4 * sizeof(uint32_t), s));
-  if (m) k_degrees<<<grid_for(m), 256, 0, s>>>(keys, m, deg_u, deg_v);
+  if (m) k_degrees<<<grid_for(m), 256, 0, s>>>(keys, m, deg_u, deg_v), gmbe_note_launch();
   unsigned long long *okeys, *okeys2;
   TRY(t.alloc(&okeys, NV));
   TRY(t.alloc(&okeys2, NV));
-  if (NV) k_order_keys<<<grid_for(NV), 256, 0, s>>>(deg_v, NV, o.order == GMBE_ORDER_IDENTITY, okeys);
+  if (NV) k_order_keys<<<grid_for(NV), 256, 0, s>>>(deg_v, NV, o.order == GMBE_ORDER_IDENTITY, okeys), gmbe_note_launch();
   TRY(radix_sort(t, okeys, okeys2, NV, 32 + bits_for(m + 1), s));
   // persistent buffers
   uint32_t *off_v, *adj_v, *off_u, *adj_u, *rank2id;
@@ -277,20 +290,20 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   // library V side == caller V (hash side 1) unless swapped (then caller U, side 0)
   if (NV)
     k_rank_maps<<<grid_for(NV), 256, 0, s>>>(okeys2, NV, swapped ? 0u : 1u, rank2id, id2rank, deg_v,
-                                             deg_by_rank, hv);
+                                             deg_by_rank, hv), gmbe_note_launch();
   TRY(excl_scan(t, deg_by_rank, off_v, (uint64_t)NV + 1, s));
   TRY(excl_scan(t, deg_u, off_u, (uint64_t)NU + 1, s));
   if (m) {
     unsigned long long *kv, *ku;
     TRY(t.alloc(&kv, m));
     TRY(t.alloc(&ku, m));
-    k_rekey<<<grid_for(m), 256, 0, s>>>(keys, m, id2rank, kv, ku);
+    k_rekey<<<grid_for(m), 256, 0, s>>>(keys, m, id2rank, kv, ku), gmbe_note_launch();
     TRY(radix_sort(t, kv, keys2, m, 32 + bits_for(NV), s));
-    k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_v);
+    k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_v), gmbe_note_launch();
     TRY(radix_sort(t, ku, keys2, m, 32 + bits_for(NU), s));
-    k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_u);
+    k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_u), gmbe_note_launch();
   }
-  if (NV || NU) k_bounds<<<grid_for((uint64_t)NV * 32 + NU), 256, 0, s>>>(off_v, adj_v, off_u, NV, NU, maxes);
+  if (NV || NU) k_bounds<<<grid_for((uint64_t)NV * 32 + NU), 256, 0, s>>>(off_v, adj_v, off_u, NV, NU, maxes), gmbe_note_launch();
   TRY(cudaGetLastError());
   uint32_t hm[4];
   TRY(cudaMemcpyAsync(hm, maxes, sizeof(hm), cudaMemcpyDeviceToHost, s));
@@ -341,8 +354,8 @@ extern "C" void gmbe_free_graph(gmbe_graph* G) {
   cudaGetDevice(&prev);
   cudaSetDevice(G->device);
   cudaStreamSynchronize(G->stream);
-  gmbe_release_workspace(G);
-  for (int i = 0; i < G->nbufs; i++) cudaFree(G->bufs[i]);
+  for (int i = 0; i < G->nbufs; i++) cudaFreeAsync(G->bufs[i], G->stream);
+  cudaStreamSynchronize(G->stream);
   if (G->own_stream) cudaStreamDestroy(G->stream);
   cudaSetDevice(prev);
   delete G;

@@ -38,8 +38,8 @@ struct gmbe_graph {
   int nbufs;
 };
 
-// workspace cache of gmbe_enumerate, freed with the graph (gmbe_enum.cu)
-extern "C" void gmbe_release_workspace(const gmbe_graph* g);
+// count of this library's own kernel launches (gmbe_api.cu)
+void gmbe_note_launch();
 
 // thread-local error plumbing (gmbe_api.cu)
 int gmbe_set_error(int code, const std::string& msg);
