@@ -96,7 +96,8 @@ typedef struct {
                                output, so counts / checksums add (mod 2^64) across parts */
   uint32_t counters;      /* 1: also compute nodes/nonmax-exact algo_bytes (slower; no early
                                exit in the maximality scan).  nodes / nonmax are always exact. */
-  uint32_t reserved0;
+  uint32_t wedge_l;       /* roots with |L_r| > wedge_l generate their children from the wedges of L'
+                             and rebase them; 0 = default 64, max 64 */
   /* Optional bounded output (device-accessible memory: device or mapped pinned host).
    * Record = [|L|, |R|, L ids (caller U ids), R ids (caller V ids)], order within a record and of
    * records unspecified; out_offsets[i] = word offset of record i in out_ids.  A full buffer is
@@ -109,7 +110,8 @@ typedef struct {
   /* Optional per-root counts (HOST memory, length = library-internal |V|): bicliques emitted under
    * each root vertex, indexed by the root's caller id on the library's V side. */
   uint64_t* per_root_count;
-  /* Workspace (0 = auto): words of the per-warp node stack arena; words / number of task slabs. */
+  /* Workspace (0 = auto): words of the per-warp dynamic region (root record, node stack); words
+   * per task slab and number of slabs. */
   uint64_t arena_words;
   uint64_t slab_words;
   uint64_t n_slabs;

@@ -28,6 +28,9 @@ namespace {
 constexpr uint32_t kHdr = 8;  // node record header words
 constexpr uint32_t kNone = 0xffffffffu;
 constexpr uint32_t kPruned = 0x80000000u;
+constexpr uint32_t kRTag = 0xfffffffeu;   // table value of an R vertex (wedge mode)
+constexpr uint32_t kClaim = 0xfffffffdu;  // slotmap placeholder while a slot is claimed
+constexpr uint32_t kSmemSort = 256;       // per-warp shared-memory sort capacity (keys)
 
 struct Ctrl {
   unsigned long long root_cursor, q_head, q_tail, f_head, f_tail, pending;
@@ -44,8 +47,10 @@ struct Params {
   uint32_t part_index, part_count;
   uint32_t prune, split, bound_height, bound_size, counters;
   uint32_t hu_side;   // checksum side of the library's U vertices (0 = caller U)
-  uint32_t* arena;
+  uint32_t wedge_l;    // roots with |L_r| > wedge_l use wedge-mode child generation
+  uint32_t* arena;    // per warp: keys[tmax] | slotmap[emax] | vals[tmax] (u64) | occ[omax] | dynamic
   uint64_t arena_words;
+  uint32_t tmax, emax, omax;
   uint32_t* rbuf;     // per-warp R-list stack (only with output)
   uint32_t rbuf_words;
   uint32_t* slabs;
@@ -570,220 +575,187 @@ __device__ void dispatch_task(const Params& P, const TaskCtx& T, uint32_t* top, 
   else run_task<32>(P, T, top, lo, hi, lmap, A);
 }
 
-// ---------------------------------------------------------------- root task (a3)
-__device__ void run_root(const Params& P, uint32_t r, uint32_t* arena, uint32_t* rbuf, Acc& A) {
+// ---------------------------------------------------------------- small warp sorts
+// sort n 64-bit keys in a[0..n) ascending; a has room for next_pow2(n) keys.
+__device__ void warp_sort_keys(unsigned long long* a, uint32_t n, unsigned long long* smem) {
   const uint32_t lane = lane_id();
-  const DevGraph& g = P.g;
-  const uint32_t lb = g.off_v[r], l = g.off_v[r + 1] - lb;
-  if (l == 0) return;  // isolated vertex: in no biclique (A17)
-  const uint32_t* Lr = g.adj_v + lb;
-  // wedge count (and the root's algorithmic bytes)
-  uint32_t wp = 0;
-  for (uint32_t j = lane; j < l; j += 32) {
-    uint32_t u = Lr[j];
-    wp += g.off_u[u + 1] - g.off_u[u];
-  }
-  const uint32_t wedges = warp_sum(wp);
-  if (P.counters) {
-    A.abytes += 4ull * (l + wedges);
-    A.aqfull += 4ull * (l + wedges);
-  }
-  uint32_t T = next_pow2(max(64u, 2u * wedges));
-  const uint32_t logT = 31 - __clz(T);
-  const uint32_t shift = 32 - logT, mask = T - 1;
-  uint32_t* keys = arena;
-  uint32_t* vals = arena + T;
-  if (2ull * T + 64 > P.arena_words) {
-    if (lane == 0) atomicOr(&P.ctrl->error, kErrArena);
-    return;
-  }
-  for (uint32_t j = lane; j < T; j += 32) {
-    keys[j] = GMBE_EMPTY;
-    vals[j] = 0;
-  }
-  __syncwarp();
-  __threadfence_block();
-  const bool small = l <= 32;  // rows fit one word: build them directly in pass 1
-  // pass 1: N2(v_s) with local neighbourhood sizes k(v_c) = |N(v_c) ∩ L_r| (Alg 3 L2-3)
-  for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
-    if (act && v != r) {
-      uint32_t h = ht_insert(keys, shift, mask, v);
-      if (small) atomicOr(vals + h, 1u << i);
-      else atomicAdd(vals + h, 1u);
-    }
-  });
-  __syncwarp();
-  __threadfence();
-  // scan 1: classify.  k == |L| -> R (skip root unless v_s is the earliest in R, Alg 3 L7),
-  // later-ordered -> C, earlier-ordered -> Q.
-  uint32_t nC = 0, nQ = 0, nR = 0;
-  bool skip = false;
-  unsigned long long sr = 0;
-  for (uint32_t b = 0; b < T; b += 32) {
-    const uint32_t s = b + lane;
-    const uint32_t v = __ldcg(keys + s);
-    const bool occ = v != GMBE_EMPTY;
-    uint32_t c = 0;
-    if (occ) {
-      uint32_t x = __ldcg(vals + s);
-      c = small ? __popc(x) : x;
-    }
-    const bool isR = occ && c == l;
-    skip |= isR && v < r;
-    const bool isC = occ && !isR && v > r;
-    const bool isQ = occ && !isR && v < r;
-    if (isR) sr += g.hv[v];
-    const uint32_t bR = __ballot_sync(GMBE_FULL, isR);
-    if (rbuf && isR) rbuf[1 + nR + __popc(bR & lanemask_lt())] = v;
-    nR += __popc(bR);
-    nC += __popc(__ballot_sync(GMBE_FULL, isC));
-    nQ += __popc(__ballot_sync(GMBE_FULL, isQ));
-  }
-  if (__any_sync(GMBE_FULL, skip)) {
-    __syncwarp();
-    return;
-  }
-  A.roots_run++;
-  sr = warp_sum64(sr) + g.hv[r];
-  // emit (L_r, R_r)  (A5)
-  {
-    unsigned long long sl = 0;
-    for (uint32_t j = lane; j < l; j += 32) sl += hash_u(P, Lr[j]);
-    sl = warp_sum64(sl);
-    A.count++;
-    A.checksum += pair_hash(P, sl, sr);
-    if (P.per_root && lane == 0) atomicAdd(P.per_root + r, 1ull);
-    if (rbuf) {
-      if (lane == 0) rbuf[0] = r;
-      __syncwarp();
-      if (P.out_ids) write_record(P, nullptr, 0, nullptr, Lr, l, rbuf, nR + 1);
-    }
-  }
-  if (nC == 0) return;
-
-  // ---- build the root node record.  Scratch after the table: sort buffer | useful bits |
-  // useful-word prefix | compacted map | root record | DFS stack.
-  uint32_t* scratch = vals + T;
-  unsigned long long* sortbuf = (unsigned long long*)(((uintptr_t)scratch + 15) & ~(uintptr_t)15);
-  uint32_t* after_sort = (uint32_t*)(sortbuf + next_pow2(nC));
-  const uint32_t nuw = (l + 31) / 32;
-  uint32_t* useful = after_sort;        // l bits (large roots)
-  uint32_t* upre = useful + r4(nuw);    // exclusive prefix popcount of useful words
-  uint32_t* mapbuf = upre + r4(nuw);    // compacted universe
-  uint32_t* rec = (uint32_t*)(((uintptr_t)(small ? after_sort : mapbuf + r4(l)) + 15) & ~(uintptr_t)15);
-  {
-    const uint64_t wmax = (l + 31) / 32;
-    const uint64_t need = (uint64_t)(rec - arena) + kHdr + r4(wmax) + (uint64_t)(nC + nQ) * r4(wmax + 2) + 64;
-    if (need > P.arena_words) {
-      if (lane == 0) atomicOr(&P.ctrl->error, kErrArena);
-      return;
-    }
-  }
-  uint32_t lu = l;                 // universe size
-  const uint32_t* map = Lr;        // universe map
-  if (!small) {
-    // pass 2: keep only L_r vertices adjacent to some candidate (every child L' lies inside)
-    for (uint32_t j = lane; j < nuw; j += 32) useful[j] = 0;
-    __syncwarp();
-    for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
-      if (act && v > r) {
-        uint32_t h = ht_find(keys, shift, mask, v);
-        if (h != kNone && __ldcg(vals + h) < l) atomicOr(useful + (i >> 5), 1u << (i & 31));
+  if (n <= 1) return;
+  if (n <= 32) {  // register bitonic network over the warp
+    unsigned long long x = lane < n ? a[lane] : ~0ull;
+#pragma unroll
+    for (uint32_t k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+      for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+        unsigned long long y = __shfl_xor_sync(GMBE_FULL, x, j);
+        const bool up = (lane & k) == 0;
+        const bool lower = (lane & j) == 0;
+        x = (lower == up) ? (x < y ? x : y) : (x < y ? y : x);
       }
-    });
-    __syncwarp();
-    __threadfence();
-    uint32_t c = 0;
-    for (uint32_t b = 0; b < l; b += 32) {
-      const uint32_t i = b + lane;
-      const uint32_t uw = __ldcg(useful + (b >> 5));
-      if (lane == 0) upre[b >> 5] = c;
-      const bool u = i < l && ((uw >> lane) & 1u);
-      const uint32_t bal = __ballot_sync(GMBE_FULL, u);
-      if (u) mapbuf[c + __popc(bal & lanemask_lt())] = Lr[i];
-      c += __popc(bal);
     }
-    lu = c;
-    map = mapbuf;
     __syncwarp();
+    if (lane < n) a[lane] = x;
+    __syncwarp();
+    return;
   }
+  if (next_pow2(n) <= kSmemSort) {  // bitonic in this warp's shared-memory slice
+    for (uint32_t j = lane; j < n; j += 32) smem[j] = a[j];
+    __syncwarp();
+    warp_sort64(smem, n);
+    for (uint32_t j = lane; j < n; j += 32) a[j] = smem[j];
+    __syncwarp();
+    return;
+  }
+  warp_sort64(a, n);
+}
+
+// warp-cooperative insert of v (lanes with act) into the per-warp table; new slots are appended
+// to occ (so the table can be cleaned in O(occupied)).  Returns the slot.
+__device__ __forceinline__ uint32_t ht_insert_warp(uint32_t* keys, uint32_t shift, uint32_t mask, uint32_t v,
+                                                   bool act, uint32_t* occ, uint32_t& nocc) {
+  uint32_t h = act ? ht_hash(v, shift) : 0, slot = kNone;
+  bool pend = act;
+  while (__any_sync(GMBE_FULL, pend)) {
+    bool ins = false;
+    if (pend) {
+      const uint32_t k = __ldcg(keys + h);
+      if (k == v) {
+        slot = h;
+        pend = false;
+      } else if (k == GMBE_EMPTY) {
+        const uint32_t old = atomicCAS(keys + h, GMBE_EMPTY, v);
+        if (old == GMBE_EMPTY || old == v) {
+          slot = h;
+          pend = false;
+          ins = old == GMBE_EMPTY;
+        } else {
+          h = (h + 1) & mask;
+        }
+      } else {
+        h = (h + 1) & mask;
+      }
+    }
+    const uint32_t b = __ballot_sync(GMBE_FULL, ins);
+    if (ins) occ[nocc + __popc(b & lanemask_lt())] = h;
+    nocc += __popc(b);
+  }
+  return slot;
+}
+
+// Per-warp memory: a persistently clean hash table (keys EMPTY, vals 0), its occupied-slot list,
+// the entry->child-slot map (NONE), and the dynamic region (records, scratch, node stack).
+struct WarpMem {
+  uint32_t* keys;
+  uint32_t* slotmap;
+  unsigned long long* vals;
+  uint32_t* occ;
+  uint32_t* dyn;
+  uint32_t* dyn_end;
+  uint32_t* rbuf;
+  unsigned long long* sm_sort;  // shared-memory sort slice
+};
+
+__device__ __forceinline__ uint32_t* align4(uint32_t* p) {
+  return (uint32_t*)(((uintptr_t)p + 15) & ~(uintptr_t)15);
+}
+
+__device__ __forceinline__ bool fits(const Params& P, const uint32_t* p, const uint32_t* end) {
+  if (p <= end) return true;
+  if (lane_id() == 0) atomicOr(&P.ctrl->error, kErrArena);
+  return false;
+}
+
+// Copy a self-contained task (universe map + R list + node record) into a free slab and enqueue
+// it (Alg 4 L25).  Returns false if no slab is free or the task does not fit one.
+__device__ bool enqueue_record(const Params& P, const uint32_t* map, uint32_t lmap, uint32_t W, uint32_t root,
+                               const uint32_t* rlist, uint32_t rlen, const uint32_t* rec, uint32_t words,
+                               Acc& A) {
+  const uint32_t lane = lane_id();
+  const uint32_t node_off = slab_node_off(lmap, rlist ? rlen : 0);
+  if (node_off + words > P.slab_words) return false;
+  const uint32_t slab = slab_alloc(P);
+  if (slab == kNone) return false;
+  uint32_t* s = P.slabs + (uint64_t)slab * P.slab_words;
+  for (uint32_t j = lane; j < lmap; j += 32) s[kHdr + j] = map[j];
+  if (rlist)
+    for (uint32_t j = lane; j < rlen; j += 32) s[kHdr + r4(lmap) + j] = rlist[j];
+  for (uint32_t j = lane; j < words; j += 32) s[node_off + j] = rec[j];
+  if (lane == 0) {
+    s[0] = W;
+    s[1] = lmap;
+    s[2] = root;
+    s[3] = rlist ? rlen : 0;
+    s[4] = node_off;
+  }
+  A.tasks++;
+  __threadfence();
+  __syncwarp();
+  if (lane == 0) {
+    atomicAdd(&P.ctrl->pending, 1ull);
+    ring_push(P.tq, P.ring_mask, &P.ctrl->q_tail, slab);
+  }
+  return true;
+}
+
+__device__ __forceinline__ bool heavy(const Params& P, uint32_t l, uint32_t nC) {
+  const unsigned long long h = min(l, nC);  // tree height estimate
+  return P.split && h > P.bound_height && h * nC > P.bound_size;
+}
+
+// ---------------------------------------------------------------- root record, bitmap mode
+// |L_r| <= wedge_l (<= 64): rows N(x) ∩ L_r (one or two words) come straight from the table.
+__device__ void bitmap_root(const Params& P, uint32_t r, uint32_t l, const uint32_t* Lr, uint32_t nC, uint32_t nQ,
+                            uint32_t nR, unsigned long long sr, uint32_t nocc, WarpMem& M, Acc& A) {
+  const uint32_t lane = lane_id();
   TaskCtx Tc;
-  Tc.map = map;
-  Tc.W = (lu + 31) / 32;
+  Tc.map = Lr;
+  Tc.W = (l + 31) / 32;
   Tc.W4 = r4(Tc.W);
   Tc.E = r4(Tc.W + 2);
   Tc.root = r;
-  Tc.rlist = rbuf;
-  const uint64_t rec_need = kHdr + Tc.W4 + (uint64_t)(nC + nQ) * Tc.E;
-  uint32_t* ent = rec + kHdr + Tc.W4;
+  Tc.rlist = M.rbuf;
   const uint32_t W = Tc.W, E = Tc.E;
-  // zero rows of the large-root entries (filled by pass 3)
-  if (!small)
-    for (uint64_t j = lane; j < (uint64_t)(nC + nQ) * E; j += 32) ent[j] = 0;
-  __syncwarp();
-  // scan 2: C -> sort buffer, Q -> entries nC.. (table order)
-  {
-    uint32_t cc = 0, qc = 0;
-    for (uint32_t b = 0; b < T; b += 32) {
-      const uint32_t s = b + lane;
-      const uint32_t v = __ldcg(keys + s);
-      const bool occ = v != GMBE_EMPTY;
-      uint32_t x = occ ? __ldcg(vals + s) : 0;
-      const uint32_t c = small ? __popc(x) : x;
-      const bool isR = occ && c == l;
-      const bool isC = occ && !isR && v > r;
-      const bool isQ = occ && !isR && v < r;
-      const uint32_t bC = __ballot_sync(GMBE_FULL, isC);
-      if (isC) sortbuf[cc + __popc(bC & lanemask_lt())] = ((unsigned long long)v << 32) | s;
-      cc += __popc(bC);
-      const uint32_t bQ = __ballot_sync(GMBE_FULL, isQ);
-      if (isQ) {
-        const uint32_t e = nC + qc + __popc(bQ & lanemask_lt());
-        uint32_t* ee = ent + (size_t)e * E;
-        if (small) ee[0] = x;
-        ee[W] = v;
-        ee[W + 1] = c;
-        if (!small) vals[s] = e;
-      }
-      qc += __popc(bQ);
-      if (!small && isR) vals[s] = kNone;
+  unsigned long long* sortbuf = (unsigned long long*)align4(M.dyn);
+  uint32_t* rec = align4((uint32_t*)(sortbuf + next_pow2(nC)));
+  const uint64_t rec_need = kHdr + Tc.W4 + (uint64_t)(nC + nQ) * E;
+  if (!fits(P, rec + rec_need + 64, M.dyn_end)) return;
+  uint32_t* ent = rec + kHdr + Tc.W4;
+  uint32_t cc = 0, qc = 0;
+  for (uint32_t b = 0; b < nocc; b += 32) {
+    const uint32_t j = b + lane;
+    const bool occ = j < nocc;
+    const uint32_t s = occ ? M.occ[j] : 0;
+    const uint32_t v = occ ? __ldcg(M.keys + s) : 0;
+    const unsigned long long x = occ ? __ldcg(M.vals + s) : 0;
+    const uint32_t c = __popcll(x);
+    const bool isR = occ && c == l;
+    const bool isC = occ && !isR && v > r;
+    const bool isQ = occ && !isR && v < r;
+    const uint32_t bC = __ballot_sync(GMBE_FULL, isC);
+    if (isC) sortbuf[cc + __popc(bC & lanemask_lt())] = ((unsigned long long)v << 32) | s;
+    cc += __popc(bC);
+    const uint32_t bQ = __ballot_sync(GMBE_FULL, isQ);
+    if (isQ) {
+      uint32_t* ee = ent + (size_t)(nC + qc + __popc(bQ & lanemask_lt())) * E;
+      ee[0] = (uint32_t)x;
+      if (W == 2) ee[1] = (uint32_t)(x >> 32);
+      ee[W] = v;
+      ee[W + 1] = c;
     }
+    qc += __popc(bQ);
   }
   __syncwarp();
-  warp_sort64(sortbuf, nC);  // candidates in rank order (Alg 2 L6: smallest first)
+  warp_sort_keys(sortbuf, nC, M.sm_sort);  // candidates in rank order (Alg 2 L6)
   for (uint32_t j = lane; j < nC; j += 32) {
     const unsigned long long kv = sortbuf[j];
-    const uint32_t v = (uint32_t)(kv >> 32), s = (uint32_t)kv;
-    const uint32_t x = __ldcg(vals + s);
+    const unsigned long long x = __ldcg(M.vals + (uint32_t)kv);
     uint32_t* ee = ent + (size_t)j * E;
-    if (small) {
-      ee[0] = x;
-      ee[W + 1] = __popc(x);
-    } else {
-      ee[W + 1] = x;
-      vals[s] = j;
-    }
-    ee[W] = v;
+    ee[0] = (uint32_t)x;
+    if (W == 2) ee[1] = (uint32_t)(x >> 32);
+    ee[W] = (uint32_t)(kv >> 32);
+    ee[W + 1] = __popcll(x);
   }
-  __syncwarp();
-  __threadfence();
-  if (!small) {
-    // pass 3: rows over the compacted universe
-    for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
-      const uint32_t uw = act ? __ldcg(useful + (i >> 5)) : 0;
-      if (act && v != r && ((uw >> (i & 31)) & 1u)) {
-        const uint32_t jl = upre[i >> 5] + __popc(uw & ((1u << (i & 31)) - 1u));
-        const uint32_t h = ht_find(keys, shift, mask, v);
-        const uint32_t e = h == kNone ? kNone : __ldcg(vals + h);
-        if (e != kNone) atomicOr(ent + (size_t)e * E + (jl >> 5), 1u << (jl & 31));
-      }
-    });
-    __syncwarp();
-    __threadfence();
-  }
-  // header + L mask (all universe bits)
   for (uint32_t w = lane; w < W; w += 32) {
-    const uint32_t bits = lu - w * 32;
+    const uint32_t bits = l - w * 32;
     rec[kHdr + w] = bits >= 32 ? GMBE_FULL : ((1u << bits) - 1u);
   }
   if (lane == 0) {
@@ -797,16 +769,372 @@ __device__ void run_root(const Params& P, uint32_t r, uint32_t* arena, uint32_t*
     rec[7] = (uint32_t)(sr >> 32);
   }
   __syncwarp();
-  uint32_t* lo = rec + rec_need;
-  lo = (uint32_t*)(((uintptr_t)lo + 15) & ~(uintptr_t)15);
-  dispatch_task(P, Tc, rec, lo, arena + P.arena_words, lu, A);
+  dispatch_task(P, Tc, rec, align4(rec + rec_need), M.dyn_end, l, A);
 }
 
+// ---------------------------------------------------------------- root children, wedge mode
+// |L_r| > wedge_l: bitmap rows over L_r would cost (|C|+|Q|)·|L_r|/32 words per child.  Instead each
+// child L' = L_r ∩ N(c_i) is generated from the wedges of L' (cost Σ_{u∈L'} |N(u)|), with the
+// root's table giving every 2-hop vertex's class, and is REBASED onto its own universe L' --
+// a self-contained node that is run in place or queued as a subtask.
+__device__ void wedge_root(const Params& P, uint32_t r, uint32_t l, const uint32_t* Lr, uint32_t nC, uint32_t nQ,
+                           uint32_t nR, unsigned long long sr, uint32_t nocc, uint32_t shift, uint32_t mask,
+                           WarpMem& M, Acc& A) {
+  const uint32_t lane = lane_id();
+  const DevGraph& g = P.g;
+  const uint32_t nE = nC + nQ;
+  uint32_t* ids = M.dyn;
+  uint32_t* ks = ids + r4(nE);  // bit 31 = pruned (C entries)
+  unsigned long long* sortbuf = (unsigned long long*)align4(ks + r4(nE));
+  uint32_t* Lc = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
+  uint32_t* after_lc = align4(Lc + l);
+  if (!fits(P, after_lc + 64, M.dyn_end)) return;
+  // scan 2: entries (C sorted by rank, then Q); table value := entry index (R := kRTag)
+  {
+    uint32_t cc = 0, qc = 0;
+    for (uint32_t b = 0; b < nocc; b += 32) {
+      const uint32_t j = b + lane;
+      const bool occ = j < nocc;
+      const uint32_t s = occ ? M.occ[j] : 0;
+      const uint32_t v = occ ? __ldcg(M.keys + s) : 0;
+      const uint32_t c = occ ? (uint32_t)__ldcg(M.vals + s) : 0;
+      const bool isR = occ && c == l;
+      const bool isC = occ && !isR && v > r;
+      const bool isQ = occ && !isR && v < r;
+      if (isR) M.vals[s] = kRTag;
+      const uint32_t bC = __ballot_sync(GMBE_FULL, isC);
+      if (isC) sortbuf[cc + __popc(bC & lanemask_lt())] = ((unsigned long long)v << 32) | s;
+      cc += __popc(bC);
+      const uint32_t bQ = __ballot_sync(GMBE_FULL, isQ);
+      if (isQ) {
+        const uint32_t e = nC + qc + __popc(bQ & lanemask_lt());
+        ids[e] = v;
+        ks[e] = c;
+        M.vals[s] = e;
+      }
+      qc += __popc(bQ);
+    }
+  }
+  __syncwarp();
+  warp_sort_keys(sortbuf, nC, M.sm_sort);
+  for (uint32_t j = lane; j < nC; j += 32) {
+    const unsigned long long kv = sortbuf[j];
+    const uint32_t s = (uint32_t)kv;
+    ids[j] = (uint32_t)(kv >> 32);
+    ks[j] = (uint32_t)__ldcg(M.vals + s);
+    M.vals[s] = j;
+  }
+  __syncwarp();
+  const bool split_mode = heavy(P, l, nC);
+  if (split_mode) A.splits++;
+  const uint32_t rl0 = nR + 1;  // R-list length at the root
+  for (uint32_t i = 0; i < nC; i++) {
+    __syncwarp();
+    if (ks[i] & kPruned) continue;
+    const uint32_t c = ids[i];
+    // L' = L_r ∩ N(c)   (Alg 2 L8), both lists ascending; search the shorter in the longer
+    const uint32_t cb = g.off_v[c], cd = g.off_v[c + 1] - cb;
+    const uint32_t* Nc = g.adj_v + cb;
+    const uint32_t* As = l <= cd ? Lr : Nc;
+    const uint32_t* Bs = l <= cd ? Nc : Lr;
+    const uint32_t na = min(l, cd), nb = max(l, cd);
+    uint32_t lc = 0;
+    for (uint32_t b = 0; b < na; b += 32) {
+      const uint32_t j = b + lane;
+      bool found = false;
+      uint32_t x = 0;
+      if (j < na) {
+        x = As[j];
+        uint32_t lo = 0, hi = nb;
+        while (lo < hi) {
+          const uint32_t mid = (lo + hi) >> 1;
+          if (Bs[mid] < x) lo = mid + 1;
+          else hi = mid;
+        }
+        found = lo < nb && Bs[lo] == x;
+      }
+      const uint32_t bal = __ballot_sync(GMBE_FULL, found);
+      if (found) Lc[lc + __popc(bal & lanemask_lt())] = x;
+      lc += __popc(bal);
+    }
+    __syncwarp();
+    uint32_t wq = 0;
+    for (uint32_t j = lane; j < lc; j += 32) {
+      const uint32_t u = Lc[j];
+      wq += g.off_u[u + 1] - g.off_u[u];
+    }
+    const uint32_t wl = warp_sum(wq);
+    const uint32_t Wc = (lc + 31) / 32, Ec = r4(Wc + 2);
+    const uint32_t nTmax = min(nE, wl);
+    uint32_t* tid = after_lc;
+    uint32_t* tcnt = tid + r4(nTmax);
+    uint32_t* qlist = tcnt + r4(nTmax);
+    uint32_t* trow = qlist + r4(nTmax);
+    unsigned long long* csort = (unsigned long long*)align4(trow + (uint64_t)nTmax * Wc);
+    uint32_t* crec = align4((uint32_t*)(csort + next_pow2(max(nTmax, 1u))));
+    const uint64_t crec_need = kHdr + r4(Wc) + (uint64_t)nTmax * Ec;
+    if (!fits(P, crec + crec_need + 64, M.dyn_end)) return;
+    A.nodes++;
+    if (P.counters) {  // algorithmic bytes (before this step's Thm 4.1 marks)
+      unsigned long long lk = 0, qk = 0, qf = 0;
+      for (uint32_t e = lane; e < nE; e += 32) {
+        const uint32_t k = ks[e], kk = k & ~kPruned;
+        const bool pr = (k & kPruned) != 0;
+        if (e < nC) {
+          if (e > i && !pr) lk += kk;
+          else if (e < i && !pr) {
+            qf += kk;
+            if (kk >= lc) qk += kk;
+          }
+        } else {
+          qf += kk;
+          if (kk >= lc) qk += kk;
+        }
+      }
+      lk = warp_sum64(lk);
+      qk = warp_sum64(qk);
+      qf = warp_sum64(qf);
+      A.abytes += 4ull * (lc + lk + qk);
+      A.aqfull += 4ull * (lc + lk + qf);
+    }
+    // wedge pass over L': k'(x) = |N(x) ∩ L'| and rows over L' for every touched entry x
+    uint32_t nT = 0;
+    for_each_wedge(g, Lc, lc, [&](uint32_t j, uint32_t v, bool act) {
+      uint32_t e = kNone;
+      if (act && v != r && v != c) {
+        const uint32_t h = ht_find(M.keys, shift, mask, v);
+        const uint32_t x = (uint32_t)__ldcg(M.vals + h);
+        if (x != kRTag && !(x < nC && (ks[x] & kPruned))) e = x;
+      }
+      const bool claim = e != kNone && atomicCAS(M.slotmap + e, kNone, kClaim) == kNone;
+      const uint32_t b = __ballot_sync(GMBE_FULL, claim);
+      if (claim) {
+        const uint32_t idx = nT + __popc(b & lanemask_lt());
+        atomicExch(M.slotmap + e, idx);
+        tid[idx] = e;
+        atomicExch(tcnt + idx, 0u);
+        for (uint32_t w = 0; w < Wc; w++) atomicExch(trow + (size_t)idx * Wc + w, 0u);
+      }
+      nT += __popc(b);
+      __syncwarp();
+      if (e != kNone) {
+        const uint32_t s = __ldcg(M.slotmap + e);
+        atomicAdd(tcnt + s, 1u);
+        atomicOr(trow + (size_t)s * Wc + (j >> 5), 1u << (j & 31));
+      }
+    });
+    __syncwarp();
+    // classify touched vertices (untouched ones have k' = 0: dropped, never pruned)
+    uint32_t nCc = 0, nQc = 0, rabs = 0;
+    unsigned long long srabs = 0;
+    bool dom = false;
+    for (uint32_t b = 0; b < nT; b += 32) {
+      const uint32_t s = b + lane;
+      const bool act = s < nT;
+      const uint32_t e = act ? tid[s] : 0;
+      const uint32_t kc = act ? __ldcg(tcnt + s) : 0;
+      const bool later = act && e < nC && e > i;
+      const bool qlike = act && !later;
+      const uint32_t kp = later ? (ks[e] & ~kPruned) : 0;
+      if (later && P.prune && kc == kp) ks[e] = kp | kPruned;  // Thm 4.1
+      const bool absorb = later && kc == lc;
+      const bool cand = later && kc < lc;
+      dom |= qlike && kc == lc;
+      const uint32_t ba = __ballot_sync(GMBE_FULL, absorb);
+      if (absorb) {
+        const uint32_t id = ids[e];
+        srabs += g.hv[id];
+        if (M.rbuf) M.rbuf[rl0 + 1 + rabs + __popc(ba & lanemask_lt())] = id;
+      }
+      rabs += __popc(ba);
+      const uint32_t bc = __ballot_sync(GMBE_FULL, cand);
+      if (cand) csort[nCc + __popc(bc & lanemask_lt())] = ((unsigned long long)e << 32) | s;
+      nCc += __popc(bc);
+      const uint32_t bq = __ballot_sync(GMBE_FULL, qlike);
+      if (qlike) qlist[nQc + __popc(bq & lanemask_lt())] = s;
+      nQc += __popc(bq);
+    }
+    const bool nonmax = __any_sync(GMBE_FULL, dom);
+    if (nonmax) {
+      A.nonmax++;
+    } else {
+      // Output(L', R')
+      const unsigned long long srn = sr + g.hv[c] + warp_sum64(srabs);
+      const uint32_t rlen = rl0 + 1 + rabs;
+      unsigned long long sl = 0;
+      for (uint32_t j = lane; j < lc; j += 32) sl += hash_u(P, Lc[j]);
+      sl = warp_sum64(sl);
+      A.count++;
+      A.checksum += pair_hash(P, sl, srn);
+      if (P.per_root && lane == 0) atomicAdd(P.per_root + r, 1ull);
+      if (M.rbuf) {
+        if (lane == 0) M.rbuf[rl0] = c;
+        __syncwarp();
+        if (P.out_ids) write_record(P, nullptr, 0, nullptr, Lc, lc, M.rbuf, rlen);
+      }
+      if (nCc > 0) {
+        // the rebased child node over universe L'
+        __syncwarp();
+        warp_sort_keys(csort, nCc, M.sm_sort);
+        uint32_t* cent = crec + kHdr + r4(Wc);
+        for (uint32_t j = lane; j < nCc + nQc; j += 32) {
+          uint32_t e, s;
+          if (j < nCc) {
+            const unsigned long long kv = csort[j];
+            e = (uint32_t)(kv >> 32);
+            s = (uint32_t)kv;
+          } else {
+            s = qlist[j - nCc];
+            e = tid[s];
+          }
+          uint32_t* ee = cent + (size_t)j * Ec;
+          for (uint32_t w = 0; w < Wc; w++) ee[w] = __ldcg(trow + (size_t)s * Wc + w);
+          ee[Wc] = ids[e];
+          ee[Wc + 1] = __ldcg(tcnt + s);
+        }
+        for (uint32_t w = lane; w < Wc; w += 32) {
+          const uint32_t bits = lc - w * 32;
+          crec[kHdr + w] = bits >= 32 ? GMBE_FULL : ((1u << bits) - 1u);
+        }
+        if (lane == 0) {
+          crec[0] = nCc;
+          crec[1] = nQc;
+          crec[2] = lc;
+          crec[3] = 0;
+          crec[4] = kNone;
+          crec[5] = rlen;
+          crec[6] = (uint32_t)srn;
+          crec[7] = (uint32_t)(srn >> 32);
+        }
+        __syncwarp();
+        const uint32_t words = kHdr + r4(Wc) + (nCc + nQc) * Ec;
+        if (!(split_mode && enqueue_record(P, Lc, lc, Wc, r, M.rbuf, rlen, crec, words, A))) {
+          TaskCtx Tc;
+          Tc.map = Lc;
+          Tc.W = Wc;
+          Tc.W4 = r4(Wc);
+          Tc.E = Ec;
+          Tc.root = r;
+          Tc.rlist = M.rbuf;
+          dispatch_task(P, Tc, crec, align4(crec + words), M.dyn_end, lc, A);
+        }
+      }
+    }
+    __syncwarp();
+    for (uint32_t s = lane; s < nT; s += 32) M.slotmap[tid[s]] = kNone;
+    __syncwarp();
+  }
+}
+
+// ---------------------------------------------------------------- root task (a3)
+// Root v_s (rank r): L_r = N(v_s); wedge scan of N2(v_s) with local sizes k(v) = |N(v) ∩ L_r|.
+__device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
+  const uint32_t lane = lane_id();
+  const DevGraph& g = P.g;
+  const uint32_t lb = g.off_v[r], l = g.off_v[r + 1] - lb;
+  if (l == 0) return;  // isolated vertex: in no biclique (A17)
+  const uint32_t* Lr = g.adj_v + lb;
+  uint32_t wp = 0;
+  for (uint32_t j = lane; j < l; j += 32) {
+    const uint32_t u = Lr[j];
+    wp += g.off_u[u + 1] - g.off_u[u];
+  }
+  const uint32_t wedges = warp_sum(wp);
+  if (P.counters) {
+    A.abytes += 4ull * (l + wedges);
+    A.aqfull += 4ull * (l + wedges);
+  }
+  const uint32_t T = next_pow2(max(64u, 2u * wedges));
+  if (T > P.tmax) {
+    if (lane == 0) atomicOr(&P.ctrl->error, kErrArena);
+    return;
+  }
+  const uint32_t shift = 32 - (31 - __clz(T)), mask = T - 1;
+  uint32_t* keys = M.keys;
+  unsigned long long* vals = M.vals;
+  const bool bm = l <= P.wedge_l;  // bitmap mode: rows of <= 64 bits straight from the table
+  // pass 1 (Alg 3 L2-3)
+  uint32_t nocc = 0;
+  for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
+    const bool a = act && v != r;
+    const uint32_t h = ht_insert_warp(keys, shift, mask, v, a, M.occ, nocc);
+    if (a) {
+      if (bm) atomicOr(vals + h, 1ull << i);
+      else atomicAdd(vals + h, 1ull);
+    }
+  });
+  __syncwarp();
+  // scan 1: k == |L| -> R (skip the root unless v_s is the earliest vertex of R, Alg 3 L7),
+  // later-ordered -> C, earlier-ordered -> Q
+  uint32_t nC = 0, nQ = 0, nR = 0;
+  bool skip = false;
+  unsigned long long sr = 0;
+  for (uint32_t b = 0; b < nocc; b += 32) {
+    const uint32_t j = b + lane;
+    const bool occ = j < nocc;
+    const uint32_t s = occ ? M.occ[j] : 0;
+    const uint32_t v = occ ? __ldcg(keys + s) : 0;
+    uint32_t c = 0;
+    if (occ) {
+      const unsigned long long x = __ldcg(vals + s);
+      c = bm ? __popcll(x) : (uint32_t)x;
+    }
+    const bool isR = occ && c == l;
+    skip |= isR && v < r;
+    const bool isC = occ && !isR && v > r;
+    const bool isQ = occ && !isR && v < r;
+    if (isR) sr += g.hv[v];
+    const uint32_t bR = __ballot_sync(GMBE_FULL, isR);
+    if (M.rbuf && isR) M.rbuf[1 + nR + __popc(bR & lanemask_lt())] = v;
+    nR += __popc(bR);
+    nC += __popc(__ballot_sync(GMBE_FULL, isC));
+    nQ += __popc(__ballot_sync(GMBE_FULL, isQ));
+  }
+  skip = __any_sync(GMBE_FULL, skip);
+  if (!skip) {
+    A.roots_run++;
+    sr = warp_sum64(sr) + g.hv[r];
+    unsigned long long sl = 0;
+    for (uint32_t j = lane; j < l; j += 32) sl += hash_u(P, Lr[j]);
+    sl = warp_sum64(sl);
+    A.count++;  // emit (L_r, R_r) (A5)
+    A.checksum += pair_hash(P, sl, sr);
+    if (P.per_root && lane == 0) atomicAdd(P.per_root + r, 1ull);
+    if (M.rbuf) {
+      if (lane == 0) M.rbuf[0] = r;
+      __syncwarp();
+      if (P.out_ids) write_record(P, nullptr, 0, nullptr, Lr, l, M.rbuf, nR + 1);
+    }
+    if (nC > 0) {
+      if (bm) bitmap_root(P, r, l, Lr, nC, nQ, nR, sr, nocc, M, A);
+      else wedge_root(P, r, l, Lr, nC, nQ, nR, sr, nocc, shift, mask, M, A);
+    }
+  }
+  // leave the table clean for the next root
+  __syncwarp();
+  for (uint32_t j = lane; j < nocc; j += 32) {
+    const uint32_t s = M.occ[j];
+    keys[s] = GMBE_EMPTY;
+    vals[s] = 0;
+  }
+  __syncwarp();
+}
+
+
 __global__ void __launch_bounds__(256) k_enum(const Params P) {
+  __shared__ unsigned long long s_sort[8][kSmemSort];
   const uint32_t lane = lane_id();
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  uint32_t* arena = P.arena + (uint64_t)gw * P.arena_words;
-  uint32_t* rbuf = P.rbuf ? P.rbuf + (uint64_t)gw * P.rbuf_words : nullptr;
+  uint32_t* base = P.arena + (uint64_t)gw * P.arena_words;
+  WarpMem M;
+  M.keys = base;
+  M.slotmap = base + P.tmax;
+  M.vals = (unsigned long long*)(base + P.tmax + P.emax);
+  M.occ = base + P.tmax + P.emax + 2ull * P.tmax;
+  M.dyn = align4(M.occ + P.omax);
+  M.dyn_end = base + P.arena_words;
+  M.rbuf = P.rbuf ? P.rbuf + (uint64_t)gw * P.rbuf_words : nullptr;
+  M.sm_sort = s_sort[threadIdx.x >> 5];
   Acc A = {};
   bool roots_done = false;
   uint32_t idle = 0;
@@ -826,12 +1154,11 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       Tc.W4 = r4(Tc.W);
       Tc.E = r4(Tc.W + 2);
       Tc.map = s + kHdr;
-      Tc.rlist = rbuf;
-      if (rbuf)
-        for (uint32_t j = lane; j < rlen; j += 32) rbuf[j] = s[kHdr + r4(lmap) + j];
+      Tc.rlist = M.rbuf;
+      if (M.rbuf)
+        for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
       __syncwarp();
-      uint32_t* top = s + s[4];
-      dispatch_task(P, Tc, top, arena, arena + P.arena_words, lmap, A);
+      dispatch_task(P, Tc, s + s[4], M.dyn, M.dyn_end, lmap, A);
       __syncwarp();
       slab_free(P, task);
       if (lane == 0) atomicAdd(&P.ctrl->pending, ~0ull);
@@ -848,7 +1175,7 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       t = __shfl_sync(GMBE_FULL, t, 0);
       if (t < P.n_roots) {
         const uint32_t j = P.n_roots - 1 - (uint32_t)t;
-        run_root(P, P.part_index + j * P.part_count, arena, rbuf, A);
+        run_root(P, P.part_index + j * P.part_count, M, A);
         __syncwarp();
         if (lane == 0) atomicAdd(&P.ctrl->pending, ~0ull);
         idle = 0;
@@ -891,6 +1218,8 @@ struct Workspace {
   int device = -1;
   void* arena = nullptr;
   size_t arena_bytes = 0;
+  uint64_t layout[5] = {0, 0, 0, 0, 0};  // tmax, emax, omax, arena_words, nwarps of the clean tables
+  bool clean = false;
   void* slabs = nullptr;
   size_t slab_bytes = 0;
   void* rings = nullptr;
@@ -953,21 +1282,23 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   const uint32_t blocks = (uint32_t)sms * bps;
   const uint64_t nwarps = (uint64_t)blocks * 8;
 
-  // arena sizing: hash table + root record + stack for the worst root (bounded by memory)
-  const uint64_t wb = g.wedge_bound + 64;
-  const uint64_t Tmax = 1ull << (64 - __builtin_clzll(2 * wb));
-  const uint64_t Wmax = (g.delta_v + 31) / 32;
-  const uint64_t Emax = (Wmax + 2 + 3) & ~3ull;
-  uint64_t arena_words = o.arena_words;
-  if (!arena_words) {
-    uint64_t want = 2 * Tmax + 2 * Tmax /*sort*/ + 4 * wb + wb * Emax * 3 + (1u << 16);
+  // per-warp arena: clean hash table sized for the largest root's wedges, entry map, occupied list,
+  // and the dynamic region (root record, rebased children, node stack), bounded by free memory
+  const uint64_t wb = (uint64_t)g.wedge_bound + 64;
+  uint64_t tmax = 64;
+  while (tmax < 2 * wb) tmax <<= 1;
+  const uint64_t emax = (wb + 3) & ~3ull, omax = emax;
+  const uint64_t fixed = tmax + emax + 2 * tmax + omax + 8;
+  uint64_t dyn = o.arena_words;
+  if (!dyn) {
+    const uint64_t want = 24 * wb + (1u << 18);
     size_t fr = 0, tot = 0;
     GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
-    uint64_t cap = (uint64_t)(fr * 0.45) / 4 / nwarps;
-    arena_words = want < cap ? want : cap;
-    if (arena_words < (1u << 16)) arena_words = 1u << 16;
+    const uint64_t cap_total = (uint64_t)(fr * 0.5) / 4 / nwarps;
+    const uint64_t cap = cap_total > fixed + (1u << 16) ? cap_total - fixed : (1u << 16);
+    dyn = want < cap ? want : cap;
   }
-  arena_words = (arena_words + 3) & ~3ull;
+  const uint64_t arena_words = (fixed + dyn + 3) & ~3ull;
   uint64_t slab_words = o.slab_words ? o.slab_words : (1u << 16);
   slab_words = (slab_words + 3) & ~3ull;
   uint64_t n_slabs = o.n_slabs ? o.n_slabs : 8192;
@@ -978,6 +1309,17 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   const uint32_t rbuf_words = want_out ? (uint32_t)(wb + 64) : 0;
 
   GMBE_CUDA_TRY(ensure(&W.arena, &W.arena_bytes, nwarps * arena_words * 4));
+  {
+    const uint64_t sig[5] = {tmax, emax, omax, arena_words, nwarps};
+    if (!W.clean || std::memcmp(sig, W.layout, sizeof(sig)) != 0) {
+      // keys + slotmap := 0xff.. (EMPTY / NONE), vals := 0 -- once; every root leaves them clean
+      GMBE_CUDA_TRY(cudaMemset2DAsync(W.arena, arena_words * 4, 0xff, (tmax + emax) * 4, nwarps, s));
+      GMBE_CUDA_TRY(cudaMemset2DAsync((uint32_t*)W.arena + tmax + emax, arena_words * 4, 0, 2 * tmax * 4,
+                                      nwarps, s));
+      std::memcpy(W.layout, sig, sizeof(sig));
+      W.clean = true;
+    }
+  }
   GMBE_CUDA_TRY(ensure(&W.slabs, &W.slab_bytes, n_slabs * slab_words * 4));
   GMBE_CUDA_TRY(ensure(&W.rings, &W.ring_bytes, (size_t)cap * 2 * 4));
   if (want_out) GMBE_CUDA_TRY(ensure(&W.rbuf, &W.rbuf_bytes, nwarps * rbuf_words * 4));
@@ -996,8 +1338,12 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.bound_size = o.bound_size ? o.bound_size : 1500;
   P.counters = o.counters ? 1 : 0;
   P.hu_side = g.swapped ? 1 : 0;
+  P.wedge_l = o.wedge_l ? (o.wedge_l > 64 ? 64 : o.wedge_l) : 64;
   P.arena = (uint32_t*)W.arena;
   P.arena_words = arena_words;
+  P.tmax = (uint32_t)tmax;
+  P.emax = (uint32_t)emax;
+  P.omax = (uint32_t)omax;
   P.rbuf = want_out ? (uint32_t*)W.rbuf : nullptr;
   P.rbuf_words = rbuf_words;
   P.slabs = (uint32_t*)W.slabs;
@@ -1054,6 +1400,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   out->splits = hc.splits;
   out->tasks = hc.tasks;
   out->kernel_ms = ms;
+  if (hc.error) W.clean = false;
   if (hc.error)
     return gmbe_set_error(GMBE_EINTERNAL, std::string("gmbe_enumerate: device workspace exceeded (") +
                                               ((hc.error & kErrArena) ? "arena" : "slab") +

@@ -111,9 +111,11 @@ struct Tmp {
   cudaStream_t s;
   std::vector<void*> p;
   explicit Tmp(cudaStream_t st) : s(st) {}
-  ~Tmp() {
+  ~Tmp() { free_all(); }
+  void free_all() {
     for (void* x : p)
       if (x) cudaFreeAsync(x, s);
+    p.clear();
   }
   template <class T>
   cudaError_t alloc(T** out, size_t n) {
@@ -206,7 +208,9 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   G->caller_n_v = n_v;
   G->order = o.order;
   G->nbufs = 0;
+  Tmp t(s);
   auto fail = [&](int rc) {
+    t.free_all();
     for (int i = 0; i < G->nbufs; i++) cudaFreeAsync(G->bufs[i], s);
     cudaStreamSynchronize(s);
     if (own) cudaStreamDestroy(s);
@@ -224,7 +228,6 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   const uint32_t swapped = n_u < n_v ? 1u : 0u;
   const uint32_t NU = swapped ? n_v : n_u, NV = swapped ? n_u : n_v;
   const uint64_t m0 = n_edges;
-  Tmp t(s);
   // a1: ingest
   const uint32_t* d_e = edges_uv;
   if (m0 && !o.edges_on_device) {

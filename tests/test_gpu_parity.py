@@ -73,7 +73,8 @@ def test_random_tiny_sets(gmbe):
         nu, nv, e = _rand_graph(rng)
         order = "degree" if rng.random() < 0.7 else "identity"
         prune = bool(rng.random() < 0.8)
-        r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True, counters=True)
+        wl = int(rng.choice([0, 1, 2, 4]))  # 1..4: force wedge-mode roots (rebased children)
+        r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True, counters=True, wedge_l=wl)
         o = oracle.oracle_mbe(nu, nv, e, order=order, prune=prune, records=True)
         _same(r, o)
         assert r.bicliques == sorted(o.bicliques)
@@ -88,10 +89,11 @@ def test_random_medium_dense(gmbe):
         nv = int(rng.integers(10, 60))
         p = float(rng.uniform(0.05, 0.35))
         e = np.argwhere(rng.random((nu, nv)) < p).astype(np.uint32)
-        r = _run(gmbe, nu, nv, e, counters=True)
         o = oracle.oracle_mbe(nu, nv, e)
-        _same(r, o)
-        assert (r.algo_bytes, r.algo_bytes_qfull) == (o.algo_bytes, o.algo_bytes_qfull)
+        for wl in (0, 8, 33):
+            r = _run(gmbe, nu, nv, e, counters=True, wedge_l=wl)
+            _same(r, o)
+            assert (r.algo_bytes, r.algo_bytes_qfull) == (o.algo_bytes, o.algo_bytes_qfull)
 
 
 # ---------------------------------------------------------------- closed forms / edge cases
@@ -136,8 +138,8 @@ def test_swapped_orientation_sets(gmbe):
 # ---------------------------------------------------------------- ER(40,40,.15)
 def test_er40(gmbe):
     nu, nv, e = make_config("er40")
-    for prune in (True, False):
-        r = _run(gmbe, nu, nv, e, prune=prune, records=True, counters=True)
+    for prune, wl in ((True, 0), (False, 0), (True, 1), (False, 3)):
+        r = _run(gmbe, nu, nv, e, prune=prune, records=True, counters=True, wedge_l=wl)
         o = oracle.oracle_mbe(nu, nv, e, prune=prune, records=True)
         _same(r, o)
         assert r.count == 211
@@ -164,14 +166,17 @@ def test_split_and_schedule_invariance(gmbe, dense_case):
         variants = [dict(), dict(split=False), dict(bound_height=1, bound_size=1),
                     dict(bound_height=1, bound_size=1, n_slabs=1),
                     dict(bound_height=1, bound_size=1, n_slabs=3, slab_words=4096),
-                    dict(warps_per_sm=8), dict(warps_per_sm=64)]
+                    dict(warps_per_sm=8), dict(warps_per_sm=64),
+                    dict(wedge_l=1), dict(wedge_l=1, bound_height=1, bound_size=1),
+                    dict(wedge_l=16, bound_height=2, bound_size=8, n_slabs=2)]
         for kw in variants:
             r = g.enumerate(counters=True, **kw)
             _same(r, o)
             assert r.algo_bytes == o.algo_bytes, kw
-        r = g.enumerate(bound_height=1, bound_size=1, records=True)
-        assert r.tasks > 0 and r.splits > 0
-        assert r.bicliques == sorted(o.bicliques)
+        for wl in (0, 1):
+            r = g.enumerate(bound_height=1, bound_size=1, records=True, wedge_l=wl)
+            assert r.tasks > 0 and r.splits > 0
+            assert r.bicliques == sorted(o.bicliques)
     finally:
         g.free()
 
