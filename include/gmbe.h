@@ -110,6 +110,9 @@ typedef struct {
   /* Optional per-root counts (HOST memory, length = library-internal |V|): bicliques emitted under
    * each root vertex, indexed by the root's caller id on the library's V side. */
   uint64_t* per_root_count;
+  /* Optional profiling (HOST memory, same indexing): SM clock cycles the warps spent on each root's
+   * tree (root build + in-place search + its queued subtasks). */
+  uint64_t* per_root_cycles;
   /* Workspace (0 = auto): words of the per-warp dynamic region (root record, node stack); words
    * per task slab and number of slabs. */
   uint64_t arena_words;

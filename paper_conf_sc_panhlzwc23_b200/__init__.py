@@ -46,7 +46,7 @@ class Opts(ctypes.Structure):
                 ("bound_size", _u32), ("warps_per_sm", _u32), ("part_index", _u32),
                 ("part_count", _u32), ("counters", _u32), ("wedge_l", _u32),
                 ("out_offsets", _vp), ("out_offsets_cap", _u64), ("out_ids", _vp),
-                ("out_ids_cap", _u64), ("per_root_count", _vp), ("arena_words", _u64),
+                ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("arena_words", _u64),
                 ("slab_words", _u64), ("n_slabs", _u64), ("cuda_stream", _vp)]
 
 
@@ -118,6 +118,7 @@ class Result:
     kernel_ms: float
     bicliques: list = field(default=None, repr=False)
     per_root_count: np.ndarray = field(default=None, repr=False)
+    per_root_cycles: np.ndarray = field(default=None, repr=False)
 
 
 def _stream_ptr(stream):
@@ -143,7 +144,7 @@ class Graph:
 
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), counters=False, records=False, rec_cap=1 << 16, ids_cap=1 << 22,
-                  per_root=False, arena_words=0, slab_words=0, n_slabs=0, wedge_l=0, stream=None):
+                  per_root=False, root_cycles=False, arena_words=0, slab_words=0, n_slabs=0, wedge_l=0, stream=None):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
@@ -170,6 +171,11 @@ class Graph:
             nv_int = inf["n_u"] if inf["swapped"] else inf["n_v"]
             prc = np.zeros(max(nv_int, 1), np.uint64)
             o.per_root_count = prc.ctypes.data
+        prcy = None
+        if root_cycles:
+            inf = self.info()
+            prcy = np.zeros(max(inf["n_u"] if inf["swapped"] else inf["n_v"], 1), np.uint64)
+            o.per_root_cycles = prcy.ctypes.data
         cr = CResult()
         _check(_lib.gmbe_enumerate(self._h, ctypes.byref(o), ctypes.byref(cr)))
         res = Result(**{k: getattr(cr, k) for k, _ in CResult._fields_})
@@ -177,6 +183,8 @@ class Graph:
             offs = bufs[0][: res.n_written].cpu().numpy().view(np.uint64)
             ids = bufs[1].cpu().numpy().view(np.uint32)
             res.bicliques = decode_records(offs, ids)
+        if root_cycles:
+            res.per_root_cycles = prcy
         if per_root:
             res.per_root_count = prc[: (self.info()["n_u"] if self.info()["swapped"] else self.info()["n_v"])]
         return res

@@ -65,6 +65,7 @@ struct Params {
   uint32_t* out_ids;
   uint64_t out_ids_cap;
   unsigned long long* per_root;
+  unsigned long long* per_root_cycles;
 };
 
 struct Acc {
@@ -1158,7 +1159,10 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       if (M.rbuf)
         for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
       __syncwarp();
+      const long long c0 = clock64();
       dispatch_task(P, Tc, s + s[4], M.dyn, M.dyn_end, lmap, A);
+      if (P.per_root_cycles && lane == 0)
+        atomicAdd(P.per_root_cycles + Tc.root, (unsigned long long)(clock64() - c0));
       __syncwarp();
       slab_free(P, task);
       if (lane == 0) atomicAdd(&P.ctrl->pending, ~0ull);
@@ -1175,7 +1179,10 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       t = __shfl_sync(GMBE_FULL, t, 0);
       if (t < P.n_roots) {
         const uint32_t j = P.n_roots - 1 - (uint32_t)t;
+        const long long c0 = clock64();
         run_root(P, P.part_index + j * P.part_count, M, A);
+        if (P.per_root_cycles && lane == 0)
+          atomicAdd(P.per_root_cycles + P.part_index + j * P.part_count, (unsigned long long)(clock64() - c0));
         __syncwarp();
         if (lane == 0) atomicAdd(&P.ctrl->pending, ~0ull);
         idle = 0;
@@ -1229,6 +1236,8 @@ struct Workspace {
   void* ctrl = nullptr;
   void* per_root = nullptr;
   size_t per_root_bytes = 0;
+  void* per_root_cyc = nullptr;
+  size_t per_root_cyc_bytes = 0;
 };
 
 cudaError_t ensure(void** p, size_t* have, size_t need) {
@@ -1326,6 +1335,8 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   size_t ctrl_have = W.ctrl ? sizeof(Ctrl) : 0;
   GMBE_CUDA_TRY(ensure(&W.ctrl, &ctrl_have, sizeof(Ctrl)));
   if (o.per_root_count) GMBE_CUDA_TRY(ensure(&W.per_root, &W.per_root_bytes, (size_t)(g.n_v + 1) * 8));
+  if (o.per_root_cycles)
+    GMBE_CUDA_TRY(ensure(&W.per_root_cyc, &W.per_root_cyc_bytes, (size_t)(g.n_v + 1) * 8));
 
   Params P{};
   P.g = g;
@@ -1358,6 +1369,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.out_ids = o.out_ids;
   P.out_ids_cap = want_out ? o.out_ids_cap : 0;
   P.per_root = o.per_root_count ? (unsigned long long*)W.per_root : nullptr;
+  P.per_root_cycles = o.per_root_cycles ? (unsigned long long*)W.per_root_cyc : nullptr;
 
   Ctrl hc{};
   hc.f_tail = n_slabs;
@@ -1366,6 +1378,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
                                                                                     (uint32_t)n_slabs);
   gmbe_note_launch();
   if (P.per_root) GMBE_CUDA_TRY(cudaMemsetAsync(W.per_root, 0, (size_t)(g.n_v + 1) * 8, s));
+  if (P.per_root_cycles) GMBE_CUDA_TRY(cudaMemsetAsync(W.per_root_cyc, 0, (size_t)(g.n_v + 1) * 8, s));
   GMBE_CUDA_TRY(cudaGetLastError());
   cudaEvent_t e0, e1;
   GMBE_CUDA_TRY(cudaEventCreate(&e0));
@@ -1381,12 +1394,18 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   cudaEventElapsedTime(&ms, e0, e1);
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
-  if (o.per_root_count && g.n_v) {
+  if ((o.per_root_count || o.per_root_cycles) && g.n_v) {
     std::vector<unsigned long long> pr(g.n_v);
     std::vector<uint32_t> r2i(g.n_v);
-    GMBE_CUDA_TRY(cudaMemcpy(pr.data(), W.per_root, g.n_v * 8, cudaMemcpyDeviceToHost));
     GMBE_CUDA_TRY(cudaMemcpy(r2i.data(), g.rank2id, g.n_v * 4, cudaMemcpyDeviceToHost));
-    for (uint32_t rr = 0; rr < g.n_v; rr++) o.per_root_count[r2i[rr]] = pr[rr];
+    if (o.per_root_count) {
+      GMBE_CUDA_TRY(cudaMemcpy(pr.data(), W.per_root, g.n_v * 8, cudaMemcpyDeviceToHost));
+      for (uint32_t rr = 0; rr < g.n_v; rr++) o.per_root_count[r2i[rr]] = pr[rr];
+    }
+    if (o.per_root_cycles) {
+      GMBE_CUDA_TRY(cudaMemcpy(pr.data(), W.per_root_cyc, g.n_v * 8, cudaMemcpyDeviceToHost));
+      for (uint32_t rr = 0; rr < g.n_v; rr++) o.per_root_cycles[r2i[rr]] = pr[rr];
+    }
   }
   out->count = hc.count;
   out->checksum = hc.checksum;
@@ -1441,7 +1460,7 @@ extern "C" void gmbe_release_workspace(const gmbe_graph* G) {
       i++;
       continue;
     }
-    for (void* p : {w->arena, w->slabs, w->rings, w->rbuf, w->ctrl, w->per_root})
+    for (void* p : {w->arena, w->slabs, w->rings, w->rbuf, w->ctrl, w->per_root, w->per_root_cyc})
       if (p) cudaFree(p);
     delete w;
     g_ws_idle.erase(g_ws_idle.begin() + i);
