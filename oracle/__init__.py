@@ -34,7 +34,7 @@ def build(force=False):
 class _Res(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in (
         "count", "checksum", "roots_run", "nodes", "nonmax", "algo_bytes", "algo_bytes_qfull",
-        "n_written", "ids_written", "truncated", "closure_failures")]
+        "n_written", "ids_written", "truncated", "closure_failures", "algo_bytes_cand")]
 
 
 def _load():
@@ -60,6 +60,7 @@ class OracleResult:
     algo_bytes_qfull: int
     truncated: int
     closure_failures: int
+    algo_bytes_cand: int = 0
     bicliques: list = None      # list of (tuple(L), tuple(R)) in caller ids, if requested
     per_root_count: np.ndarray = None
 
@@ -85,7 +86,8 @@ def oracle_mbe(n_u, n_v, edges, order="degree", prune=True, shard=(0, 1), check_
     if rc != 0:
         raise ValueError("oracle_mbe: invalid arguments")
     out = OracleResult(res.count, res.checksum, res.roots_run, res.nodes, res.nonmax,
-                       res.algo_bytes, res.algo_bytes_qfull, res.truncated, res.closure_failures)
+                       res.algo_bytes, res.algo_bytes_qfull, res.truncated, res.closure_failures,
+                       res.algo_bytes_cand)
     if records:
         out.bicliques = decode_records(offs[:res.n_written], ids)
     if per_root:

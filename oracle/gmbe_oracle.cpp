@@ -12,7 +12,8 @@
 //   * count and checksum = sum over bicliques of h(L,R) mod 2^64, h as frozen in DESIGN.md
 //     ("Checksum"), over the CALLER's original ids and roles.
 //   * Work counters of the canonical tree (degree order + Thm 4.1, no split): nodes, nonmax,
-//     algo_bytes, algo_bytes_qfull.
+//     algo_bytes, algo_bytes_qfull, and algo_bytes_cand = the wedge + candidate terms alone
+//     (DESIGN.md "Algorithmic bytes").
 //
 // How: the textbook set-enumeration tree of Alg 1 with an explicit excluded set Q
 // (P:377-380), first level = Alg 3 root tasks with the root check "v_s is the
@@ -81,7 +82,7 @@ struct Options {
 
 struct Result {
   uint64_t count, checksum, roots_run, nodes, nonmax, algo_bytes, algo_bytes_qfull;
-  uint64_t n_written, ids_written, truncated, closure_failures;
+  uint64_t n_written, ids_written, truncated, closure_failures, algo_bytes_cand;
 };
 
 struct Oracle {
@@ -188,6 +189,7 @@ struct Oracle {
       }
       res.algo_bytes += 4 * (words + qwords);
       res.algo_bytes_qfull += 4 * (words + qwords_full);
+      res.algo_bytes_cand += 4 * words;
       // Maximality check (Alg 2 L14 "R' == Gamma(L')"): non-maximal iff some excluded vertex is
       // adjacent to all of L'.  The subtree of a non-maximal node is skipped (A3).
       std::vector<uint32_t> qnext;
@@ -230,6 +232,7 @@ struct Oracle {
     for (uint32_t u : l) wedge_words += NU[u].size();
     res.algo_bytes += 4 * wedge_words;
     res.algo_bytes_qfull += 4 * wedge_words;
+    res.algo_bytes_cand += 4 * wedge_words;
     // N2(v_s) = ∪_{u in N(v_s)} N(u) - {v_s}
     Set n2;
     for (uint32_t u : l) n2.insert(n2.end(), NU[u].begin(), NU[u].end());
@@ -281,7 +284,7 @@ extern "C" {
 
 typedef struct {
   uint64_t count, checksum, roots_run, nodes, nonmax, algo_bytes, algo_bytes_qfull;
-  uint64_t n_written, ids_written, truncated, closure_failures;
+  uint64_t n_written, ids_written, truncated, closure_failures, algo_bytes_cand;
 } oracle_result;
 
 // Returns 0 on success, -1 on invalid arguments.
