@@ -94,10 +94,7 @@ typedef struct {
   uint32_t part_index;    /* root shard: enumerate the roots whose degree rank r satisfies */
   uint32_t part_count;    /*   r % part_count == part_index (0 = 1 part); shards partition the
                                output, so counts / checksums add (mod 2^64) across parts */
-  uint32_t counters;      /* 1: also compute nodes/nonmax-exact algo_bytes (slower; no early
-                               exit in the maximality scan).  nodes / nonmax are always exact. */
-  uint32_t wedge_l;       /* roots with |L_r| > wedge_l generate their children from the wedges of L'
-                             and rebase them; 0 = default 64, max 64 */
+  uint32_t reserved0, reserved1;  /* must be 0 */
   /* Optional bounded output (device-accessible memory: device or mapped pinned host).
    * Record = [|L|, |R|, L ids (caller U ids), R ids (caller V ids)], order within a record and of
    * records unspecified; out_offsets[i] = word offset of record i in out_ids.  A full buffer is
@@ -129,8 +126,8 @@ typedef struct {
   uint64_t roots_run;     /* roots not skipped by the Alg 3 L7 check */
   uint64_t nodes;         /* generated, unpruned child nodes (canonical tree; roots excluded) */
   uint64_t nonmax;        /* nodes failing the maximality check */
-  uint64_t algo_bytes;    /* DESIGN.md algorithmic bytes (only if opts.counters) */
-  uint64_t algo_bytes_qfull;
+  uint64_t algo_bytes_cand; /* wedge + candidate-scan algorithmic bytes of the canonical tree
+                               (the Q term is not computed on the GPU) */
   uint64_t splits;        /* nodes expanded in split mode */
   uint64_t tasks;         /* subtasks enqueued */
   double kernel_ms;       /* device time of the enumeration kernel (CUDA events) */

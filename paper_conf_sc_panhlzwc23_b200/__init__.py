@@ -44,7 +44,7 @@ class GraphInfo(ctypes.Structure):
 class Opts(ctypes.Structure):
     _fields_ = [("struct_size", _u32), ("no_prune", _u32), ("no_split", _u32), ("bound_height", _u32),
                 ("bound_size", _u32), ("warps_per_sm", _u32), ("part_index", _u32),
-                ("part_count", _u32), ("counters", _u32), ("wedge_l", _u32),
+                ("part_count", _u32), ("reserved0", _u32), ("reserved1", _u32),
                 ("out_offsets", _vp), ("out_offsets_cap", _u64), ("out_ids", _vp),
                 ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("arena_words", _u64),
                 ("slab_words", _u64), ("n_slabs", _u64), ("cuda_stream", _vp)]
@@ -52,7 +52,7 @@ class Opts(ctypes.Structure):
 
 class CResult(ctypes.Structure):
     _fields_ = [(n, _u64) for n in ("count", "checksum", "n_written", "truncated", "roots_run",
-                                     "nodes", "nonmax", "algo_bytes", "algo_bytes_qfull", "splits",
+                                     "nodes", "nonmax", "algo_bytes_cand", "splits",
                                      "tasks")] + [("kernel_ms", ctypes.c_double)]
 
 
@@ -111,8 +111,7 @@ class Result:
     roots_run: int
     nodes: int
     nonmax: int
-    algo_bytes: int
-    algo_bytes_qfull: int
+    algo_bytes_cand: int
     splits: int
     tasks: int
     kernel_ms: float
@@ -143,8 +142,8 @@ class Graph:
         return {k: getattr(gi, k) for k, _ in GraphInfo._fields_}
 
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
-                  part=(0, 1), counters=False, records=False, rec_cap=1 << 16, ids_cap=1 << 22,
-                  per_root=False, root_cycles=False, arena_words=0, slab_words=0, n_slabs=0, wedge_l=0, stream=None):
+                  part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
+                  per_root=False, root_cycles=False, arena_words=0, slab_words=0, n_slabs=0, stream=None):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
@@ -152,9 +151,7 @@ class Graph:
         o.no_split = 0 if split else 1
         o.bound_height, o.bound_size, o.warps_per_sm = bound_height, bound_size, warps_per_sm
         o.part_index, o.part_count = part
-        o.counters = 1 if counters else 0
         o.arena_words, o.slab_words, o.n_slabs = arena_words, slab_words, n_slabs
-        o.wedge_l = wedge_l
         o.cuda_stream = _stream_ptr(stream)
         bufs = None
         if records:

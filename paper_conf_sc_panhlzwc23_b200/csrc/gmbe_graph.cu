@@ -85,7 +85,8 @@ __global__ void k_low32(const unsigned long long* __restrict__ k, uint64_t m, ui
 // one warp per V rank: wedge count Σ_{u∈N(v)} |N(u)| and the maxima.
 __global__ void k_bounds(const uint32_t* __restrict__ off_v, const uint32_t* __restrict__ adj_v,
                          const uint32_t* __restrict__ off_u, uint32_t n_v, uint32_t n_u,
-                         uint32_t* __restrict__ maxes /* [0]=Δ(V) [1]=Δ(U) [2]=wedge bound */) {
+                         uint32_t* __restrict__ maxes /* [0]=Δ(V) [1]=Δ(U) [2]=wedge bound */,
+                         unsigned long long* __restrict__ rec_bound) {
   uint32_t lane = threadIdx.x & 31;
   uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   uint32_t nw = (gridDim.x * blockDim.x) >> 5;
@@ -100,6 +101,9 @@ __global__ void k_bounds(const uint32_t* __restrict__ off_v, const uint32_t* __r
     if (lane == 0) {
       atomicMax(&maxes[0], e - b);
       atomicMax(&maxes[2], (uint32_t)(s > 0xffffffffull ? 0xffffffffull : s));
+      // root record: <= s candidates, each row of ceil(deg/32) words + id + k, padded to 4
+      const unsigned long long stride = (((e - b) + 31) / 32 + 2 + 3) & ~3ull;
+      atomicMax(rec_bound, s * stride);
     }
   }
   for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < n_u; u += gridDim.x * blockDim.x)
@@ -271,6 +275,9 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   TRY(t.alloc(&deg_by_rank, NV + 1));
   TRY(t.alloc(&id2rank, NV + 1));
   TRY(t.alloc(&maxes, 4));
+  unsigned long long* d_recb;
+  TRY(t.alloc(&d_recb, 1));
+  TRY(cudaMemsetAsync(d_recb, 0, 8, s));
   TRY(cudaMemsetAsync(deg_u, 0, (NU + 1) * sizeof(uint32_t), s));
   TRY(cudaMemsetAsync(deg_v, 0, (NV + 1) * sizeof(uint32_t), s));
   TRY(cudaMemsetAsync(deg_by_rank, 0, (NV + 1) * sizeof(uint32_t), s));
@@ -306,10 +313,12 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
     TRY(radix_sort(t, ku, keys2, m, 32 + bits_for(NU), s));
     k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_u), gmbe_note_launch();
   }
-  if (NV || NU) k_bounds<<<grid_for((uint64_t)NV * 32 + NU), 256, 0, s>>>(off_v, adj_v, off_u, NV, NU, maxes), gmbe_note_launch();
+  if (NV || NU) k_bounds<<<grid_for((uint64_t)NV * 32 + NU), 256, 0, s>>>(off_v, adj_v, off_u, NV, NU, maxes, d_recb), gmbe_note_launch();
   TRY(cudaGetLastError());
   uint32_t hm[4];
   TRY(cudaMemcpyAsync(hm, maxes, sizeof(hm), cudaMemcpyDeviceToHost, s));
+  unsigned long long h_recb = 0;
+  TRY(cudaMemcpyAsync(&h_recb, d_recb, 8, cudaMemcpyDeviceToHost, s));
   TRY(cudaStreamSynchronize(s));
 
   void* keep[] = {off_v, adj_v, off_u, adj_u, rank2id, hv};
@@ -331,6 +340,7 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   g.delta_v = hm[0];
   g.delta_u = hm[1];
   g.wedge_bound = hm[2];
+  g.rec_bound = h_recb;
   *out = G;
   return GMBE_OK;
 #undef TRY

@@ -46,7 +46,8 @@ def main():
             parts = pool.map(_shard, [(name, i, n) for i in range(n)])
         nu, nv, e = make_config(name)
         st = graph_stats(nu, nv, e)
-        tot = dict(count=0, checksum=0, roots_run=0, nodes=0, nonmax=0, algo_bytes=0, algo_bytes_qfull=0)
+        tot = dict(count=0, checksum=0, roots_run=0, nodes=0, nonmax=0, algo_bytes=0, algo_bytes_qfull=0,
+                   algo_bytes_cand=0)
         for r, _ in parts:
             for k in tot:
                 tot[k] += getattr(r, k)

@@ -1,7 +1,7 @@
 """GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by element.
 
 Count and checksum must be bit-exact; on small inputs the full biclique SET must be equal; the
-canonical-tree counters (nodes, nonmax, algo_bytes) must match exactly (schedule-independent,
+canonical-tree counters (nodes, nonmax, algo_bytes_cand) must match exactly (schedule-independent,
 DESIGN.md reading A9).  Marked gpu: run on the B200 box."""
 import json
 import os
@@ -33,10 +33,10 @@ def _run(gmbe, nu, nv, e, order="degree", **kw):
         g.free()
 
 
-def _same(r, o, counters=True):
+def _same(r, o):
     assert (r.count, r.checksum) == (o.count, o.checksum)
-    if counters:
-        assert (r.roots_run, r.nodes, r.nonmax) == (o.roots_run, o.nodes, o.nonmax)
+    assert (r.roots_run, r.nodes, r.nonmax) == (o.roots_run, o.nodes, o.nonmax)
+    assert r.algo_bytes_cand == o.algo_bytes_cand
 
 
 # ---------------------------------------------------------------- paper worked example
@@ -44,12 +44,12 @@ def test_g0_sets_and_tree(gmbe):
     nu, nv, e = g0_edges()
     for order in ("identity", "degree"):
         for prune in (True, False):
-            r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True, counters=True,
+            r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True,
                      per_root=True)
             o = oracle.oracle_mbe(nu, nv, e, order=order, prune=prune, records=True, per_root=True)
             _same(r, o)
             assert r.bicliques == sorted(o.bicliques)
-            assert (r.algo_bytes, r.algo_bytes_qfull) == (o.algo_bytes, o.algo_bytes_qfull)
+            assert r.algo_bytes_cand == o.algo_bytes_cand
             assert r.per_root_count.tolist() == o.per_root_count.tolist()
     # Fig 2 / Ex 4.1: identity order, t1 pruned
     r = _run(gmbe, nu, nv, e, order="identity")
@@ -73,12 +73,11 @@ def test_random_tiny_sets(gmbe):
         nu, nv, e = _rand_graph(rng)
         order = "degree" if rng.random() < 0.7 else "identity"
         prune = bool(rng.random() < 0.8)
-        wl = int(rng.choice([0, 1, 2, 4]))  # 1..4: force wedge-mode roots (rebased children)
-        r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True, counters=True, wedge_l=wl)
+        r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True)
         o = oracle.oracle_mbe(nu, nv, e, order=order, prune=prune, records=True)
         _same(r, o)
         assert r.bicliques == sorted(o.bicliques)
-        assert r.algo_bytes == o.algo_bytes
+        assert r.algo_bytes_cand == o.algo_bytes_cand
 
 
 def test_random_medium_dense(gmbe):
@@ -90,10 +89,9 @@ def test_random_medium_dense(gmbe):
         p = float(rng.uniform(0.05, 0.35))
         e = np.argwhere(rng.random((nu, nv)) < p).astype(np.uint32)
         o = oracle.oracle_mbe(nu, nv, e)
-        for wl in (0, 8, 33):
-            r = _run(gmbe, nu, nv, e, counters=True, wedge_l=wl)
-            _same(r, o)
-            assert (r.algo_bytes, r.algo_bytes_qfull) == (o.algo_bytes, o.algo_bytes_qfull)
+        r = _run(gmbe, nu, nv, e)
+        _same(r, o)
+        assert r.algo_bytes_cand == o.algo_bytes_cand
 
 
 # ---------------------------------------------------------------- closed forms / edge cases
@@ -138,13 +136,13 @@ def test_swapped_orientation_sets(gmbe):
 # ---------------------------------------------------------------- ER(40,40,.15)
 def test_er40(gmbe):
     nu, nv, e = make_config("er40")
-    for prune, wl in ((True, 0), (False, 0), (True, 1), (False, 3)):
-        r = _run(gmbe, nu, nv, e, prune=prune, records=True, counters=True, wedge_l=wl)
+    for prune in (True, False):
+        r = _run(gmbe, nu, nv, e, prune=prune, records=True)
         o = oracle.oracle_mbe(nu, nv, e, prune=prune, records=True)
         _same(r, o)
         assert r.count == 211
         assert r.bicliques == sorted(o.bicliques)
-        assert (r.algo_bytes, r.algo_bytes_qfull) == (o.algo_bytes, o.algo_bytes_qfull)
+        assert r.algo_bytes_cand == o.algo_bytes_cand
 
 
 # ---------------------------------------------------------------- schedule freedom (A9)
@@ -167,14 +165,13 @@ def test_split_and_schedule_invariance(gmbe, dense_case):
                     dict(bound_height=1, bound_size=1, n_slabs=1),
                     dict(bound_height=1, bound_size=1, n_slabs=3, slab_words=4096),
                     dict(warps_per_sm=8), dict(warps_per_sm=64),
-                    dict(wedge_l=1), dict(wedge_l=1, bound_height=1, bound_size=1),
-                    dict(wedge_l=16, bound_height=2, bound_size=8, n_slabs=2)]
+                    dict(bound_height=2, bound_size=8, n_slabs=2), dict(arena_words=4096)]
         for kw in variants:
-            r = g.enumerate(counters=True, **kw)
+            r = g.enumerate(**kw)
             _same(r, o)
-            assert r.algo_bytes == o.algo_bytes, kw
-        for wl in (0, 1):
-            r = g.enumerate(bound_height=1, bound_size=1, records=True, wedge_l=wl)
+            assert r.algo_bytes_cand == o.algo_bytes_cand, kw
+        for nsl in (0, 2):
+            r = g.enumerate(bound_height=1, bound_size=1, records=True, n_slabs=nsl)
             assert r.tasks > 0 and r.splits > 0
             assert r.bicliques == sorted(o.bicliques)
     finally:
@@ -186,11 +183,11 @@ def test_parts_are_additive(gmbe, dense_case):
     g = gmbe.load(nu, nv, e)
     try:
         for n in (2, 3, 8):
-            rs = [g.enumerate(part=(i, n), counters=True) for i in range(n)]
+            rs = [g.enumerate(part=(i, n)) for i in range(n)]
             assert sum(x.count for x in rs) == o.count
             assert sum(x.checksum for x in rs) % (1 << 64) == o.checksum
             assert sum(x.nodes for x in rs) == o.nodes
-            assert sum(x.algo_bytes for x in rs) == o.algo_bytes
+            assert sum(x.algo_bytes_cand for x in rs) == o.algo_bytes_cand
             for i in range(n):  # per-shard parity (ownership invariant)
                 os_ = oracle.oracle_mbe(nu, nv, e, shard=(i, n))
                 assert (rs[i].count, rs[i].checksum) == (os_.count, os_.checksum)
@@ -240,11 +237,10 @@ def test_full_config_vs_oracle_golden(gmbe, name):
     nu, nv, e = make_config(name)
     g = gmbe.load(nu, nv, e)
     try:
-        r = g.enumerate(counters=True)
+        r = g.enumerate()
         assert (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16))
         assert (r.nodes, r.nonmax, r.roots_run) == (gd["nodes"], gd["nonmax"], gd["roots_run"])
-        assert (r.algo_bytes, r.algo_bytes_qfull) == (gd["algo_bytes"], gd["algo_bytes_qfull"])
-        r2 = g.enumerate()  # the bench launch configuration (no counters)
-        assert (r2.count, r2.checksum) == (r.count, r.checksum)
+        if "algo_bytes_cand" in gd:
+            assert r.algo_bytes_cand == gd["algo_bytes_cand"]
     finally:
         g.free()
