@@ -20,6 +20,7 @@
 // no excluded set is stored: maximality (Alg 2 L14, "R' == Γ(L')") is decided by
 // counting Γ(L') = ∩_{u∈L'} N(u) over N(u*) for the lowest-degree u* ∈ L' (|Γ(L')| = |R'| iff
 // maximal, since R' ⊆ Γ(L')); for |L'| = 1 this is just deg(u*) == |R'|.
+#include <algorithm>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -51,6 +52,7 @@ struct Params {
   uint32_t hu_side;   // checksum side of the library's U vertices (0 = caller U)
   uint32_t* arena;    // per warp: keys[tmax] | vals[tmax] (u64) | occ[omax] | dynamic
   uint64_t arena_words;
+  uint64_t col_budget;  // max words of a root's Γ-column store
   uint32_t tmax, omax;
   uint32_t* rbuf;     // per-warp R-list stack (only with output)
   uint32_t rbuf_words;
@@ -79,6 +81,9 @@ struct TaskCtx {
   uint32_t W, W4, E;    // words per row, padded L-mask words, entry stride
   uint32_t root;        // rank of the root vertex
   uint32_t* rlist;      // R-list stack (output only)
+  const uint32_t* cols; // Γ columns of the root: cols[j*ncw ..] = bitmap of 2-hop vertices adjacent
+  uint32_t ncw;         //   to universe vertex j (null: count Γ by binary search)
+  uint32_t colslab;     // slab holding cols when shared with split subtasks (ref-counted), or kNone
 };
 
 // per-warp memory
@@ -290,8 +295,17 @@ __device__ uint32_t slab_alloc(const Params& P) {
 __device__ void slab_free(const Params& P, uint32_t s) {
   if (lane_id() == 0) ring_push(P.fq, P.ring_mask, &P.ctrl->f_tail, s);
 }
-// slab layout: [0]=W [1]=map length [2]=root rank [3]=R length [4]=node offset [5..7] pad |
-//              map | R list | node record
+// drop one reference to a shared column slab; the last holder frees it
+__device__ void colslab_release(const Params& P, uint32_t cs) {
+  if (cs == kNone) return;
+  uint32_t last = 0;
+  if (lane_id() == 0) last = atomicSub(P.slabs + (uint64_t)cs * P.slab_words, 1u) == 1u;
+  last = __shfl_sync(GMBE_FULL, last, 0);
+  if (last) slab_free(P, cs);
+}
+// task slab layout: [0]=W [1]=map length [2]=root rank [3]=R length [4]=node offset
+//                   [5]=column slab (or kNone) [6]=column words [7] pad | map | R list | node record
+// column slab layout: [0]=reference count [1..7] pad | columns
 __device__ __forceinline__ uint32_t slab_node_off(uint32_t lmap, uint32_t rlen) { return kHdr + r4(lmap) + r4(rlen); }
 // Publish the child node already written at slab + node_off as a self-contained subtask (Alg 4 L25).
 __device__ void slab_publish(const Params& P, uint32_t slab, const TaskCtx& T, uint32_t lmap, uint32_t rlen,
@@ -307,8 +321,11 @@ __device__ void slab_publish(const Params& P, uint32_t slab, const TaskCtx& T, u
     s[2] = T.root;
     s[3] = T.rlist ? rlen : 0;
     s[4] = node_off;
+    s[5] = T.colslab;
+    s[6] = T.ncw;
     s[node_off + 3] = 0;      // next candidate
     s[node_off + 4] = kNone;  // no parent: top of its task
+    if (T.colslab != kNone) atomicAdd(P.slabs + (uint64_t)T.colslab * P.slab_words, 1u);
   }
   A.tasks++;
   __threadfence();  // release the slab contents before it becomes visible in the queue
@@ -454,6 +471,31 @@ __device__ bool gamma_is_r(const Params& P, const uint32_t* lmask, uint32_t W, c
   return count == rlen;
 }
 
+// Alg 2 L14 with the root's Γ columns: every v ∈ Γ(L') other than v_s lies in the root's 2-hop set
+// X, so |Γ(L')| = 1 + popc(AND_{j ∈ L'} col_j); maximal iff that equals |R'|.
+__device__ bool gamma_cols_is_r(const TaskCtx& T, const uint32_t* lmask, uint32_t W, uint32_t rlen) {
+  const uint32_t lane = lane_id();
+  const uint32_t need = rlen - 1;  // dominators in X that are already in R'
+  uint32_t count = 0;
+  for (uint32_t xb = 0; xb < T.ncw; xb += 32) {
+    const uint32_t xw = xb + lane;
+    uint32_t acc = xw < T.ncw ? GMBE_FULL : 0u;
+    for (uint32_t w = 0; w < W; w++) {
+      uint32_t word = lmask[w];
+      while (word) {
+        const uint32_t j = w * 32 + __ffs(word) - 1;
+        word &= word - 1;
+        if (acc) acc &= __ldg(T.cols + (size_t)j * T.ncw + xw);
+        if (!__any_sync(GMBE_FULL, acc)) break;
+      }
+      if (!__any_sync(GMBE_FULL, acc)) break;
+    }
+    count += warp_sum(__popc(acc));
+    if (count > need) return false;
+  }
+  return count == need;
+}
+
 // ---------------------------------------------------------------- child generation (a4, a5)
 // Generate the child of node `par` via its candidate i into `ch` (Alg 2 L6-16).  The parent's later
 // candidates are compacted in place (Thm 4.1 prunes removed), so par[0] shrinks.
@@ -548,7 +590,18 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   const uint32_t rlen = par[5] + 1 + r_abs;
   __syncwarp();
   unsigned long long* gscr = (unsigned long long*)align4(cent + (size_t)nCc * E);
-  if (!gamma_is_r(P, lpm, W, T.map, lc, rlen, gscr, smem)) {
+  bool maximal;
+  if (lc == 1) {  // Γ({u}) = N(u)
+    uint32_t w = 0;
+    while (!lpm[w]) w++;
+    const uint32_t u = T.map[w * 32 + __ffs(lpm[w]) - 1];
+    maximal = P.g.off_u[u + 1] - P.g.off_u[u] == rlen;
+  } else if (T.cols) {
+    maximal = gamma_cols_is_r(T, lpm, W, rlen);
+  } else {
+    maximal = gamma_is_r(P, lpm, W, T.map, lc, rlen, gscr, smem);
+  }
+  if (!maximal) {
     A.nonmax++;
     return 0;
   }
@@ -724,7 +777,11 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
     nC += __popc(bC);
   }
   skip = __any_sync(GMBE_FULL, skip);
-  uint32_t* rec = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
+  // Γ columns over the 2-hop set X (= the occupied table slots; x = position in occ)
+  const uint32_t ncw = (nocc + 31) / 32;
+  uint32_t* cols = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
+  const bool want_cols = !skip && nC > 0 && (uint64_t)l * ncw <= P.col_budget;
+  uint32_t* rec = align4(cols + (want_cols ? (size_t)l * ncw : 0));
   const uint64_t rec_need = kHdr + W4 + (uint64_t)nC * E;
   if (sort_fits && !skip && fits(P, rec + rec_need + 64, M.dyn_end)) {
     A.roots_run++;
@@ -739,6 +796,24 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       if (lane == 0) M.rbuf[0] = r;
       __syncwarp();
       if (P.out_ids) write_record(P, nullptr, 0, nullptr, Lr, l, M.rbuf, nR + 1);
+    }
+    if (want_cols && small) {
+      // transpose the table rows (<= 64 bits) into columns with ballots
+      for (uint32_t b = 0; b < nocc; b += 32) {
+        const uint32_t x = b + lane;
+        const unsigned long long row = x < nocc ? __ldcg(vals + M.occ[x]) : 0ull;
+        uint32_t mine0 = 0, mine1 = 0;
+        for (uint32_t j = 0; j < l; j++) {
+          const uint32_t bal = __ballot_sync(GMBE_FULL, (row >> j) & 1ull);
+          if (lane == (j & 31)) {
+            if (j < 32) mine0 = bal;
+            else mine1 = bal;
+          }
+        }
+        if (lane < l) cols[(size_t)lane * ncw + (b >> 5)] = mine0;
+        if (lane + 32 < l) cols[(size_t)(lane + 32) * ncw + (b >> 5)] = mine1;
+      }
+      __syncwarp();
     }
     if (nC > 0) {
       // root node record: candidates in rank order (Alg 2 L6 "smallest first")
@@ -763,16 +838,26 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       }
       __syncwarp();
       if (!small) {
-        // pass 2: candidate rows over L_r
+        // pass 2: candidate rows over L_r, and the Γ columns: table value := x << 32 | C tag + entry
+        for (uint32_t x = lane; x < nocc; x += 32) {
+          const uint32_t s2 = M.occ[x];
+          const unsigned long long v2 = __ldcg(vals + s2);
+          vals[s2] = ((unsigned long long)x << 32) | ((v2 & kCTag) ? (0x80000000ull | (uint32_t)v2) : 0ull);
+        }
+        if (want_cols)
+          for (uint64_t j = lane; j < (uint64_t)l * ncw; j += 32) cols[j] = 0;
+        __syncwarp();
         for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
-          if (act && v > r) {
+          if (act && v != r) {
             const uint32_t h = ht_find(keys, shift, mask, v);
             const unsigned long long x = __ldcg(vals + h);
-            if (x & kCTag) atomicOr(ent + (size_t)(uint32_t)x * E + (i >> 5), 1u << (i & 31));
+            const uint32_t xi = (uint32_t)(x >> 32);
+            if (want_cols) atomicOr(cols + (size_t)i * ncw + (xi >> 5), 1u << (xi & 31));
+            if (x & 0x80000000ull) atomicOr(ent + (size_t)(x & 0x7fffffffull) * E + (i >> 5), 1u << (i & 31));
           }
         });
         __syncwarp();
-        __threadfence();  // rows were built with atomics: drop stale L1 lines before plain loads
+        __threadfence();  // rows / columns were built with atomics: drop stale L1 lines
       }
       for (uint32_t w = lane; w < W; w += 32) {
         const uint32_t bits = l - w * 32;
@@ -796,7 +881,24 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       Tc.E = E;
       Tc.root = r;
       Tc.rlist = M.rbuf;
+      Tc.cols = want_cols ? cols : nullptr;
+      Tc.ncw = ncw;
+      Tc.colslab = kNone;
+      if (want_cols && heavy(P, l, nC) && kHdr + (uint64_t)l * ncw <= P.slab_words) {
+        // the root will be split: share its columns with the subtasks through a ref-counted slab
+        const uint32_t cs = slab_alloc(P);
+        if (cs != kNone) {
+          uint32_t* csp = P.slabs + (uint64_t)cs * P.slab_words;
+          for (uint64_t j = lane; j < (uint64_t)l * ncw; j += 32) csp[kHdr + j] = cols[j];
+          if (lane == 0) csp[0] = 1;
+          __threadfence();
+          __syncwarp();
+          Tc.cols = csp + kHdr;
+          Tc.colslab = cs;
+        }
+      }
       dispatch_task(P, Tc, rec, align4(rec + rec_need), M.dyn_end, l, A, M.sm_sort);
+      colslab_release(P, Tc.colslab);
     }
   }
   // leave the table clean for the next root
@@ -842,6 +944,9 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       Tc.E = r4(Tc.W + 2);
       Tc.map = s + kHdr;
       Tc.rlist = M.rbuf;
+      Tc.colslab = s[5];
+      Tc.ncw = s[6];
+      Tc.cols = Tc.colslab != kNone ? P.slabs + (uint64_t)Tc.colslab * P.slab_words + kHdr : nullptr;
       if (M.rbuf)
         for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
       __syncwarp();
@@ -850,6 +955,7 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       if (P.per_root_cycles && lane == 0)
         atomicAdd(P.per_root_cycles + Tc.root, (unsigned long long)(clock64() - c0));
       __syncwarp();
+      colslab_release(P, Tc.colslab);
       slab_free(P, task);
       if (lane == 0) atomicAdd(&P.ctrl->pending, ~0ull);
       idle = 0;
@@ -1026,7 +1132,9 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   const uint64_t fixed = 3 * tmax + omax + 8;
   uint64_t dyn = o.arena_words;
   if (!dyn) {
-    const uint64_t want = (uint64_t)g.rec_bound * 4 + 4 * wb + (1u << 18);
+    // root record + node stack + Γ columns (|L_r| x |X|/32, capped at 2M words)
+    const uint64_t cols_bound = std::min<uint64_t>((uint64_t)g.delta_v * (wb / 32 + 1), 1u << 21);
+    const uint64_t want = (uint64_t)g.rec_bound * 4 + 4 * wb + 2 * cols_bound + (1u << 18);
     size_t fr = 0, tot = 0;
     GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
     const uint64_t cap_total = (uint64_t)(fr * 0.5) / 4 / nwarps;
@@ -1073,6 +1181,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.hu_side = g.swapped ? 1 : 0;
   P.arena = (uint32_t*)W.arena;
   P.arena_words = arena_words;
+  P.col_budget = dyn / 2;
   P.tmax = (uint32_t)tmax;
   P.omax = (uint32_t)omax;
   P.rbuf = want_out ? (uint32_t*)W.rbuf : nullptr;
