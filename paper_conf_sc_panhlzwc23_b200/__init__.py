@@ -23,6 +23,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 GMBE_OK, GMBE_EINVAL, GMBE_ENOMEM, GMBE_ECUDA, GMBE_EUNSUPPORTED, GMBE_EINTERNAL = 0, -1, -2, -3, -4, -5
 ORDER = {"degree": 0, "identity": 1}
+PHASES = ("root_wedges", "classify", "sort", "root_record", "cand_scan", "maximality", "emit", "queue")
 EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmbe_node_buf_bound_bytes",
            "gmbe_kernel_launch_count",
            "gmbe_naive_alloc_bytes", "gmbe_enumerate", "gmbe_release_workspace", "gmbe_last_error")
@@ -46,7 +47,7 @@ class Opts(ctypes.Structure):
                 ("bound_size", _u32), ("warps_per_sm", _u32), ("part_index", _u32),
                 ("part_count", _u32), ("reserved0", _u32), ("reserved1", _u32),
                 ("out_offsets", _vp), ("out_offsets_cap", _u64), ("out_ids", _vp),
-                ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("arena_words", _u64),
+                ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("phase_cycles", _vp), ("arena_words", _u64),
                 ("slab_words", _u64), ("n_slabs", _u64), ("cuda_stream", _vp)]
 
 
@@ -118,6 +119,7 @@ class Result:
     bicliques: list = field(default=None, repr=False)
     per_root_count: np.ndarray = field(default=None, repr=False)
     per_root_cycles: np.ndarray = field(default=None, repr=False)
+    phase_cycles: dict = field(default=None, repr=False)
 
 
 def _stream_ptr(stream):
@@ -143,7 +145,7 @@ class Graph:
 
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
-                  per_root=False, root_cycles=False, arena_words=0, slab_words=0, n_slabs=0, stream=None):
+                  per_root=False, root_cycles=False, phases=False, arena_words=0, slab_words=0, n_slabs=0, stream=None):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
@@ -173,6 +175,10 @@ class Graph:
             inf = self.info()
             prcy = np.zeros(max(inf["n_u"] if inf["swapped"] else inf["n_v"], 1), np.uint64)
             o.per_root_cycles = prcy.ctypes.data
+        phc = None
+        if phases:
+            phc = np.zeros(8, np.uint64)
+            o.phase_cycles = phc.ctypes.data
         cr = CResult()
         _check(_lib.gmbe_enumerate(self._h, ctypes.byref(o), ctypes.byref(cr)))
         res = Result(**{k: getattr(cr, k) for k, _ in CResult._fields_})
@@ -182,6 +188,8 @@ class Graph:
             res.bicliques = decode_records(offs, ids)
         if root_cycles:
             res.per_root_cycles = prcy
+        if phases:
+            res.phase_cycles = dict(zip(PHASES, phc.tolist()))
         if per_root:
             res.per_root_count = prc[: (self.info()["n_u"] if self.info()["swapped"] else self.info()["n_v"])]
         return res

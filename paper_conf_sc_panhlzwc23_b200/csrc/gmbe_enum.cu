@@ -39,6 +39,7 @@ struct Ctrl {
   unsigned long long root_cursor, q_head, q_tail, f_head, f_tail, pending;
   unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
   unsigned long long out_rec, out_ids;
+  unsigned long long phase[8];
   unsigned int truncated, error;
 };
 
@@ -69,11 +70,24 @@ struct Params {
   uint64_t out_ids_cap;
   unsigned long long* per_root;
   unsigned long long* per_root_cycles;
+  uint32_t profile;
 };
 
 struct Acc {
   unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
+  unsigned long long ph[8];  // profiling: SM cycles per phase (opts.phase_cycles)
+  long long t0;
 };
+// phase profiling (no-op unless P.profile): 0 root wedge pass, 1 classify, 2 sort, 3 root record +
+// columns, 4 candidate scan, 5 maximality, 6 emit, 7 task queue
+#define PH_START(A) \
+  if (P.profile) (A).t0 = clock64()
+#define PH_STOP(A, k)                                   \
+  if (P.profile) {                                      \
+    const long long _t = clock64();                     \
+    (A).ph[k] += (unsigned long long)(_t - (A).t0);     \
+    (A).t0 = _t;                                        \
+  }
 
 // per-task constants (warp-uniform)
 struct TaskCtx {
@@ -527,6 +541,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   __syncwarp();
   const uint32_t* lpm = ch + kHdr;  // L' words (W > LPE only)
 
+  PH_START(A);
   // later candidates: k' (Alg 2 L9-13), Thm 4.1 pruning with in-place compaction of
   // the survivors, absorption into R' (k' = |L'|), C' (0 < k' < |L'|)
   uint32_t nCc = 0, nsurv = 0, r_abs = 0;
@@ -590,6 +605,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   const uint32_t rlen = par[5] + 1 + r_abs;
   __syncwarp();
   unsigned long long* gscr = (unsigned long long*)align4(cent + (size_t)nCc * E);
+  PH_STOP(A, 4);
   bool maximal;
   if (lc == 1) {  // Γ({u}) = N(u)
     uint32_t w = 0;
@@ -601,6 +617,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   } else {
     maximal = gamma_is_r(P, lpm, W, T.map, lc, rlen, gscr, smem);
   }
+  PH_STOP(A, 5);
   if (!maximal) {
     A.nonmax++;
     return 0;
@@ -622,6 +639,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
     __syncwarp();
     if (P.out_ids) write_record(P, lpm, W, T.map, nullptr, lc, T.rlist, rlen);
   }
+  PH_STOP(A, 6);
   if (nCc == 0) return 1;
   if (lane == 0) {
     ch[0] = nCc;
@@ -686,8 +704,10 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     }
     const int r = gen_child<LPE>(P, T, cur, i, ch, A, smem);
     if (slab != kNone) {
+      PH_START(A);
       if (r == 2) slab_publish(P, slab, T, lmap, T.rlist ? ch[5] : 0, node_off, A);
       else slab_free(P, slab);
+      PH_STOP(A, 7);
       continue;
     }
     if (r == 2) {  // push (Alg 2 L16)
@@ -736,6 +756,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
   uint32_t* keys = M.keys;
   unsigned long long* vals = M.vals;
   const bool small = l <= 64;  // rows (<= 64 bits) straight from the table
+  PH_START(A);
   // pass 1 (Alg 3 L2-3)
   uint32_t nocc = 0;
   for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
@@ -747,6 +768,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
     }
   });
   __syncwarp();
+  PH_STOP(A, 0);
   // classify: k == |L| -> R (root skipped unless v_s is the earliest vertex of R, Alg 3 L7);
   // later-ordered partial neighbours -> C (Alg 3 L5-6); earlier-ordered ones are never candidates
   unsigned long long* sortbuf = (unsigned long long*)align4(M.dyn);
@@ -777,6 +799,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
     nC += __popc(bC);
   }
   skip = __any_sync(GMBE_FULL, skip);
+  PH_STOP(A, 1);
   // Γ columns over the 2-hop set X (= the occupied table slots; x = position in occ)
   const uint32_t ncw = (nocc + 31) / 32;
   uint32_t* cols = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
@@ -818,7 +841,9 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
     if (nC > 0) {
       // root node record: candidates in rank order (Alg 2 L6 "smallest first")
       __syncwarp();
+      PH_STOP(A, 3);
       warp_sort_keys(sortbuf, nC, M.sm_sort);
+      PH_STOP(A, 2);
       uint32_t* ent = rec + kHdr + W4;
       for (uint32_t j = lane; j < nC; j += 32) {
         const unsigned long long kv = sortbuf[j];
@@ -897,6 +922,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
           Tc.colslab = cs;
         }
       }
+      PH_STOP(A, 3);
       dispatch_task(P, Tc, rec, align4(rec + rec_need), M.dyn_end, l, A, M.sm_sort);
       colslab_release(P, Tc.colslab);
     }
@@ -1001,6 +1027,8 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
     atomicAdd(&c->abytes, A.abytes);
     atomicAdd(&c->splits, A.splits);
     atomicAdd(&c->tasks, A.tasks);
+    if (P.profile)
+      for (int k = 0; k < 8; k++) atomicAdd(&c->phase[k], A.ph[k]);
   }
 }
 
@@ -1199,6 +1227,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.out_ids_cap = want_out ? o.out_ids_cap : 0;
   P.per_root = o.per_root_count ? (unsigned long long*)W.per_root : nullptr;
   P.per_root_cycles = o.per_root_cycles ? (unsigned long long*)W.per_root_cyc : nullptr;
+  P.profile = o.phase_cycles ? 1 : 0;
 
   Ctrl hc{};
   hc.f_tail = n_slabs;
@@ -1246,6 +1275,8 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   out->splits = hc.splits;
   out->tasks = hc.tasks;
   out->kernel_ms = ms;
+  if (o.phase_cycles)
+    for (int k = 0; k < 8; k++) o.phase_cycles[k] = hc.phase[k];
   if (hc.error) {
     W.clean = false;
     return gmbe_set_error(GMBE_EINTERNAL,

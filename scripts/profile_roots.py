@@ -22,7 +22,7 @@ for a in sys.argv[2:]:
 nu, nv, e = make_config(name)
 g = gmbe.load(nu, nv, e)
 g.enumerate(**kw)
-r = g.enumerate(root_cycles=True, per_root=True, **kw)
+r = g.enumerate(root_cycles=True, per_root=True, phases=True, **kw)
 cyc = r.per_root_cycles.astype(np.float64)
 deg = np.bincount(e[:, 1].astype(np.int64), minlength=nv) if nu >= nv else np.bincount(e[:, 0].astype(np.int64), minlength=nu)
 order = np.argsort(-cyc)
@@ -30,5 +30,8 @@ tot = cyc.sum()
 print(json.dumps(dict(config=name, kernel_ms=r.kernel_ms, count=r.count, total_cycles=tot,
                       max_root_cycles=float(cyc.max()), ms_at_1965=float(cyc.max()) / 1.965e6,
                       top1pct_share=float(np.sort(cyc)[::-1][: max(1, len(cyc) // 100)].sum() / tot))))
+tp = sum(r.phase_cycles.values()) or 1
+print("phases:", {k: "%.1f%%" % (100.0 * v / tp) for k, v in r.phase_cycles.items()}, "profiled/total %.2f" % (tp / tot))
+print("nodes", r.nodes, "nonmax", r.nonmax, "splits", r.splits, "tasks", r.tasks)
 for v in order[:top]:
     print("root %d deg %d cycles %.3g (%.2f ms) bicliques %d" % (v, deg[v], cyc[v], cyc[v] / 1.965e6, r.per_root_count[v]))
