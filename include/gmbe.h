@@ -110,9 +110,8 @@ typedef struct {
   /* Optional profiling (HOST memory, same indexing): SM clock cycles the warps spent on each root's
    * tree (root build + in-place search + its queued subtasks). */
   uint64_t* per_root_cycles;
-  /* Optional profiling (HOST uint64_t[8]): SM cycles summed over warps per phase: root wedge pass,
-   * classification, candidate sort, root record + Γ columns, candidate scan, maximality check,
-   * emission, task queue. */
+  /* Optional profiling (HOST uint64_t[16]): SM cycles summed over warps per phase (names in the
+   * Python binding's PHASES). */
   uint64_t* phase_cycles;
   /* Workspace (0 = auto): words of the per-warp dynamic region (root record, node stack); words
    * per task slab and number of slabs. */

@@ -23,7 +23,8 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 GMBE_OK, GMBE_EINVAL, GMBE_ENOMEM, GMBE_ECUDA, GMBE_EUNSUPPORTED, GMBE_EINTERNAL = 0, -1, -2, -3, -4, -5
 ORDER = {"degree": 0, "identity": 1}
-PHASES = ("root_wedges", "classify", "sort", "root_record", "cand_scan", "maximality", "emit", "queue")
+PHASES = ("root_wedges", "classify", "sort", "root_finish", "cand_scan", "maximality", "emit", "queue",
+          "root_emit", "col_transpose", "root_entries", "root_pass2", "root_mask_hdr", "", "", "")
 EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmbe_node_buf_bound_bytes",
            "gmbe_kernel_launch_count",
            "gmbe_naive_alloc_bytes", "gmbe_enumerate", "gmbe_release_workspace", "gmbe_last_error")
@@ -177,7 +178,7 @@ class Graph:
             o.per_root_cycles = prcy.ctypes.data
         phc = None
         if phases:
-            phc = np.zeros(8, np.uint64)
+            phc = np.zeros(16, np.uint64)
             o.phase_cycles = phc.ctypes.data
         cr = CResult()
         _check(_lib.gmbe_enumerate(self._h, ctypes.byref(o), ctypes.byref(cr)))

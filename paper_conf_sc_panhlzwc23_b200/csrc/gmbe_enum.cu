@@ -39,7 +39,7 @@ struct Ctrl {
   unsigned long long root_cursor, q_head, q_tail, f_head, f_tail, pending;
   unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
   unsigned long long out_rec, out_ids;
-  unsigned long long phase[8];
+  unsigned long long phase[16];
   unsigned int truncated, error;
 };
 
@@ -75,7 +75,7 @@ struct Params {
 
 struct Acc {
   unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
-  unsigned long long ph[8];  // profiling: SM cycles per phase (opts.phase_cycles)
+  unsigned long long ph[16];  // profiling: SM cycles per phase (opts.phase_cycles)
   long long t0;
 };
 // phase profiling (no-op unless P.profile): 0 root wedge pass, 1 classify, 2 sort, 3 root record +
@@ -820,6 +820,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       __syncwarp();
       if (P.out_ids) write_record(P, nullptr, 0, nullptr, Lr, l, M.rbuf, nR + 1);
     }
+    PH_STOP(A, 8);
     if (want_cols && small) {
       // transpose the table rows (<= 64 bits) into columns with ballots
       for (uint32_t b = 0; b < nocc; b += 32) {
@@ -838,6 +839,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       }
       __syncwarp();
     }
+    PH_STOP(A, 9);
     if (nC > 0) {
       // root node record: candidates in rank order (Alg 2 L6 "smallest first")
       __syncwarp();
@@ -862,6 +864,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
         ee[W] = (uint32_t)(kv >> 32);
       }
       __syncwarp();
+      PH_STOP(A, 10);
       if (!small) {
         // pass 2: candidate rows over L_r, and the Γ columns: table value := x << 32 | C tag + entry
         for (uint32_t x = lane; x < nocc; x += 32) {
@@ -884,6 +887,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
         __syncwarp();
         __threadfence();  // rows / columns were built with atomics: drop stale L1 lines
       }
+      PH_STOP(A, 11);
       for (uint32_t w = lane; w < W; w += 32) {
         const uint32_t bits = l - w * 32;
         rec[kHdr + w] = bits >= 32 ? GMBE_FULL : ((1u << bits) - 1u);
@@ -909,6 +913,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       Tc.cols = want_cols ? cols : nullptr;
       Tc.ncw = ncw;
       Tc.colslab = kNone;
+      PH_STOP(A, 12);
       if (want_cols && heavy(P, l, nC) && kHdr + (uint64_t)l * ncw <= P.slab_words) {
         // the root will be split: share its columns with the subtasks through a ref-counted slab
         const uint32_t cs = slab_alloc(P);
@@ -1028,7 +1033,7 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
     atomicAdd(&c->splits, A.splits);
     atomicAdd(&c->tasks, A.tasks);
     if (P.profile)
-      for (int k = 0; k < 8; k++) atomicAdd(&c->phase[k], A.ph[k]);
+      for (int k = 0; k < 16; k++) atomicAdd(&c->phase[k], A.ph[k]);
   }
 }
 
@@ -1276,7 +1281,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   out->tasks = hc.tasks;
   out->kernel_ms = ms;
   if (o.phase_cycles)
-    for (int k = 0; k < 8; k++) o.phase_cycles[k] = hc.phase[k];
+    for (int k = 0; k < 16; k++) o.phase_cycles[k] = hc.phase[k];
   if (hc.error) {
     W.clean = false;
     return gmbe_set_error(GMBE_EINTERNAL,
