@@ -23,7 +23,7 @@ sys.path.insert(0, ROOT)
 
 DEFAULT_CONFIG = "gh_work"
 METRIC = "maximal bicliques/sec (Github-shaped)"
-CTRL_D2H_BYTES = 144  # sizeof(Ctrl) read back by gmbe_enumerate (gmbe_enum.cu)
+CTRL_D2H_BYTES = 1024  # sizeof(Ctrl) read back by gmbe_enumerate (static_assert in gmbe_enum.cu)
 
 
 def _args():

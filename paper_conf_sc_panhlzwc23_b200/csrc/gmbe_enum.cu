@@ -35,13 +35,21 @@ constexpr uint32_t kNone = 0xffffffffu;
 constexpr uint32_t kSmemSort = 256;  // per-warp shared-memory sort capacity (keys)
 constexpr unsigned long long kCTag = 1ull << 63;  // table value tag of a candidate (entry index)
 
+// Control block: every hot atomic on its own 128-byte line, so polling warps do not serialise the
+// atomics of working warps.
+struct alignas(128) Line {
+  unsigned long long v;
+  unsigned long long pad[15];
+};
 struct Ctrl {
-  unsigned long long root_cursor, q_head, q_tail, f_head, f_tail, pending;
+  Line root_cursor, q_head, q_tail, f_head, f_tail, pending;
   unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
   unsigned long long out_rec, out_ids;
   unsigned long long phase[16];
   unsigned int truncated, error;
 };
+
+static_assert(sizeof(Ctrl) == 1024, "bench.py reports sizeof(Ctrl) as the per-step D2H bytes");
 
 enum : unsigned int { kErrArena = 1 };
 
@@ -303,11 +311,11 @@ __device__ uint32_t ring_pop(uint32_t* ring, uint32_t mask, unsigned long long* 
 }
 __device__ uint32_t slab_alloc(const Params& P) {
   uint32_t s = kNone;
-  if (lane_id() == 0) s = ring_pop(P.fq, P.ring_mask, &P.ctrl->f_head, &P.ctrl->f_tail);
+  if (lane_id() == 0) s = ring_pop(P.fq, P.ring_mask, &P.ctrl->f_head.v, &P.ctrl->f_tail.v);
   return __shfl_sync(GMBE_FULL, s, 0);
 }
 __device__ void slab_free(const Params& P, uint32_t s) {
-  if (lane_id() == 0) ring_push(P.fq, P.ring_mask, &P.ctrl->f_tail, s);
+  if (lane_id() == 0) ring_push(P.fq, P.ring_mask, &P.ctrl->f_tail.v, s);
 }
 // drop one reference to a shared column slab; the last holder frees it
 __device__ void colslab_release(const Params& P, uint32_t cs) {
@@ -345,8 +353,8 @@ __device__ void slab_publish(const Params& P, uint32_t slab, const TaskCtx& T, u
   __threadfence();  // release the slab contents before it becomes visible in the queue
   __syncwarp();
   if (lane == 0) {
-    atomicAdd(&P.ctrl->pending, 1ull);
-    ring_push(P.tq, P.ring_mask, &P.ctrl->q_tail, slab);
+    atomicAdd(&P.ctrl->pending.v, 1ull);
+    ring_push(P.tq, P.ring_mask, &P.ctrl->q_tail.v, slab);
   }
 }
 
@@ -961,7 +969,7 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
   while (true) {
     // 1. split subtasks first (Alg 4 L3-4)
     uint32_t task = kNone;
-    if (lane == 0) task = ring_pop(P.tq, P.ring_mask, &P.ctrl->q_head, &P.ctrl->q_tail);
+    if (lane == 0) task = ring_pop(P.tq, P.ring_mask, &P.ctrl->q_head.v, &P.ctrl->q_tail.v);
     task = __shfl_sync(GMBE_FULL, task, 0);
     if (task != kNone) {
       __threadfence();  // acquire: the slab was written on another SM
@@ -988,7 +996,7 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       __syncwarp();
       colslab_release(P, Tc.colslab);
       slab_free(P, task);
-      if (lane == 0) atomicAdd(&P.ctrl->pending, ~0ull);
+      if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
       idle = 0;
       continue;
     }
@@ -996,8 +1004,8 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
     if (!roots_done) {
       unsigned long long t = 0;
       if (lane == 0) {
-        atomicAdd(&P.ctrl->pending, 1ull);
-        t = atomicAdd(&P.ctrl->root_cursor, 1ull);
+        atomicAdd(&P.ctrl->pending.v, 1ull);
+        t = atomicAdd(&P.ctrl->root_cursor.v, 1ull);
       }
       t = __shfl_sync(GMBE_FULL, t, 0);
       if (t < P.n_roots) {
@@ -1007,19 +1015,19 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
         if (P.per_root_cycles && lane == 0)
           atomicAdd(P.per_root_cycles + rk, (unsigned long long)(clock64() - c0));
         __syncwarp();
-        if (lane == 0) atomicAdd(&P.ctrl->pending, ~0ull);
+        if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
         idle = 0;
         continue;
       }
-      if (lane == 0) atomicAdd(&P.ctrl->pending, ~0ull);
+      if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
       roots_done = true;
     }
     // 3. termination: all roots issued and nothing queued or running
     unsigned long long pend = 0;
-    if (lane == 0) pend = ld_volatile(&P.ctrl->pending);
+    if (lane == 0) pend = ld_volatile(&P.ctrl->pending.v);
     pend = __shfl_sync(GMBE_FULL, pend, 0);
     if (pend == 0) break;
-    __nanosleep(idle < 8 ? 256 : 2048);
+    __nanosleep(idle < 4 ? 500 : (idle < 16 ? 2000 : 8000));  // exponential-ish backoff
     idle++;
   }
   if (lane == 0) {
@@ -1235,7 +1243,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.profile = o.phase_cycles ? 1 : 0;
 
   Ctrl hc{};
-  hc.f_tail = n_slabs;
+  hc.f_tail.v = n_slabs;
   GMBE_CUDA_TRY(cudaMemcpyAsync(W.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
   k_init_rings<<<(cap + 255) / 256 < 1024 ? (cap + 255) / 256 : 1024, 256, 0, s>>>(P.tq, P.fq, cap, (uint32_t)n_slabs);
   gmbe_note_launch();
