@@ -24,7 +24,8 @@ _lib = ctypes.CDLL(LIB_PATH)
 GMBE_OK, GMBE_EINVAL, GMBE_ENOMEM, GMBE_ECUDA, GMBE_EUNSUPPORTED, GMBE_EINTERNAL = 0, -1, -2, -3, -4, -5
 ORDER = {"degree": 0, "identity": 1}
 PHASES = ("root_wedges", "classify", "sort", "root_finish", "cand_scan", "maximality", "emit", "queue",
-          "root_emit", "col_transpose", "root_entries", "root_pass2", "root_mask_hdr", "", "", "")
+          "root_emit", "col_transpose", "root_entries", "root_pass2", "root_mask_hdr", "slab_alloc",
+          "lprime", "dequeue")
 EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmbe_node_buf_bound_bytes",
            "gmbe_kernel_launch_count",
            "gmbe_naive_alloc_bytes", "gmbe_enumerate", "gmbe_release_workspace", "gmbe_last_error")
@@ -146,7 +147,7 @@ class Graph:
 
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
-                  per_root=False, root_cycles=False, phases=False, arena_words=0, slab_words=0, n_slabs=0, stream=None):
+                  per_root=False, root_cycles=False, phases=False, debug=0, arena_words=0, slab_words=0, n_slabs=0, stream=None):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
@@ -156,6 +157,7 @@ class Graph:
         o.part_index, o.part_count = part
         o.arena_words, o.slab_words, o.n_slabs = arena_words, slab_words, n_slabs
         o.cuda_stream = _stream_ptr(stream)
+        o.reserved0 = debug
         bufs = None
         if records:
             import torch

@@ -79,6 +79,7 @@ struct Params {
   unsigned long long* per_root;
   unsigned long long* per_root_cycles;
   uint32_t profile;
+  uint32_t debug;  // opts.reserved0 bits (experiments): 1 = no shared column slabs
 };
 
 struct Acc {
@@ -297,11 +298,15 @@ __device__ void ring_push(uint32_t* ring, uint32_t mask, unsigned long long* tai
 }
 // called by one lane; returns kNone if empty
 __device__ uint32_t ring_pop(uint32_t* ring, uint32_t mask, unsigned long long* head, unsigned long long* tail) {
+  uint32_t backoff = 32;
   while (true) {
     const unsigned long long h = ld_volatile(head);
     const unsigned long long t = ld_volatile(tail);
     if (h >= t) return kNone;
-    if (atomicCAS(head, h, h + 1) == h) {
+    if (atomicCAS(head, h, h + 1) != h) {  // lost the race: back off before retrying
+      __nanosleep(backoff + (clock() & 63));
+      backoff = min(backoff * 2, 4096u);
+    } else {
       uint32_t* slot = ring + (h & mask);
       uint32_t x;
       while ((x = atomicExch(slot, GMBE_EMPTY)) == GMBE_EMPTY) __nanosleep(32);
@@ -535,6 +540,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   uint32_t* cent = ch + kHdr + T.W4;
   const uint32_t* vrow = pent + (size_t)i * E;
   const uint32_t vid = vrow[W];
+  PH_START(A);
   // L' = L_p ∩ N(v')   (Alg 2 L8)
   uint32_t lpart = 0, xw = 0;
   for (uint32_t w = lane; w < W; w += 32) {
@@ -548,8 +554,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   if (sub >= W) lp0 = 0;
   __syncwarp();
   const uint32_t* lpm = ch + kHdr;  // L' words (W > LPE only)
-
-  PH_START(A);
+  PH_STOP(A, 14);
   // later candidates: k' (Alg 2 L9-13), Thm 4.1 pruning with in-place compaction of
   // the survivors, absorption into R' (k' = |L'|), C' (0 < k' < |L'|)
   uint32_t nCc = 0, nsurv = 0, r_abs = 0;
@@ -694,29 +699,26 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     if (lane == 0) cur[3] = i + 1;
     // child record bound: later candidates + the Γ-check scratch
     const uint64_t need = kHdr + T.W4 + (uint64_t)(cur[0] - i - 1) * T.E + 4ull * 32 * T.W + 16;
-    uint32_t slab = kNone;
-    uint32_t node_off = 0;
-    const bool to_queue = split_mode && cur == top;
-    const bool stack_ok = sp + need <= stack_hi;
-    if (to_queue || !stack_ok) {
-      const uint32_t rlen_max = T.rlist ? cur[5] + 1 + cur[0] : 0;
-      node_off = slab_node_off(lmap, rlen_max);
-      if (node_off + need <= P.slab_words) slab = slab_alloc(P);
-    }
-    uint32_t* ch;
-    if (slab != kNone) {
-      ch = P.slabs + (uint64_t)slab * P.slab_words + node_off;
-    } else {
-      if (!fits(P, sp + need, stack_hi)) return;
-      ch = sp;
-    }
+    if (!fits(P, sp + need, stack_hi)) return;
+    uint32_t* ch = sp;  // children are generated on this warp's stack; only a published one is copied
     const int r = gen_child<LPE>(P, T, cur, i, ch, A, smem);
-    if (slab != kNone) {
+    if (r == 2 && split_mode && cur == top) {
+      // Alg 4 L25: hand the child to the task queue as a self-contained subtask
       PH_START(A);
-      if (r == 2) slab_publish(P, slab, T, lmap, T.rlist ? ch[5] : 0, node_off, A);
-      else slab_free(P, slab);
-      PH_STOP(A, 7);
-      continue;
+      const uint32_t words = rec_words(T, ch);
+      const uint32_t rlen = T.rlist ? ch[5] : 0;
+      const uint32_t node_off = slab_node_off(lmap, rlen);
+      uint32_t slab = kNone;
+      if (node_off + words <= P.slab_words) slab = slab_alloc(P);
+      PH_STOP(A, 13);
+      if (slab != kNone) {
+        uint32_t* dst = P.slabs + (uint64_t)slab * P.slab_words + node_off;
+        for (uint32_t j = lane; j < words; j += 32) dst[j] = ch[j];
+        __syncwarp();
+        slab_publish(P, slab, T, lmap, rlen, node_off, A);
+        PH_STOP(A, 7);
+        continue;
+      }
     }
     if (r == 2) {  // push (Alg 2 L16)
       if (lane == 0) {
@@ -922,7 +924,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       Tc.ncw = ncw;
       Tc.colslab = kNone;
       PH_STOP(A, 12);
-      if (want_cols && heavy(P, l, nC) && kHdr + (uint64_t)l * ncw <= P.slab_words) {
+      if (!(P.debug & 1) && want_cols && heavy(P, l, nC) && kHdr + (uint64_t)l * ncw <= P.slab_words) {
         // the root will be split: share its columns with the subtasks through a ref-counted slab
         const uint32_t cs = slab_alloc(P);
         if (cs != kNone) {
@@ -972,6 +974,7 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
     if (lane == 0) task = ring_pop(P.tq, P.ring_mask, &P.ctrl->q_head.v, &P.ctrl->q_tail.v);
     task = __shfl_sync(GMBE_FULL, task, 0);
     if (task != kNone) {
+      PH_START(A);
       __threadfence();  // acquire: the slab was written on another SM
       uint32_t* s = P.slabs + (uint64_t)task * P.slab_words;
       TaskCtx Tc;
@@ -989,6 +992,7 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       if (M.rbuf)
         for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
       __syncwarp();
+      PH_STOP(A, 15);
       const long long c0 = clock64();
       dispatch_task(P, Tc, s + s[4], M.dyn, M.dyn_end, lmap, A, M.sm_sort);
       if (P.per_root_cycles && lane == 0)
@@ -1241,6 +1245,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.per_root = o.per_root_count ? (unsigned long long*)W.per_root : nullptr;
   P.per_root_cycles = o.per_root_cycles ? (unsigned long long*)W.per_root_cyc : nullptr;
   P.profile = o.phase_cycles ? 1 : 0;
+  P.debug = o.reserved0;
 
   Ctrl hc{};
   hc.f_tail.v = n_slabs;
