@@ -114,10 +114,11 @@ typedef struct {
    * Python binding's PHASES). */
   uint64_t* phase_cycles;
   /* Workspace (0 = auto): words of the per-warp dynamic region (root record, node stack); words
-   * per task slab and number of slabs. */
+   * of the task pool (split subtasks and shared Γ columns; when it is exhausted work simply stays
+   * with the warp that generated it); capacity of the task queue (entries). */
   uint64_t arena_words;
-  uint64_t slab_words;
-  uint64_t n_slabs;
+  uint64_t pool_words;
+  uint64_t queue_cap;
   void* cuda_stream;      /* NULL = the graph's stream */
 } gmbe_opts;
 

@@ -24,7 +24,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 GMBE_OK, GMBE_EINVAL, GMBE_ENOMEM, GMBE_ECUDA, GMBE_EUNSUPPORTED, GMBE_EINTERNAL = 0, -1, -2, -3, -4, -5
 ORDER = {"degree": 0, "identity": 1}
 PHASES = ("root_wedges", "classify", "sort", "root_finish", "cand_scan", "maximality", "emit", "queue",
-          "root_emit", "col_transpose", "root_entries", "root_pass2", "root_mask_hdr", "slab_alloc",
+          "root_emit", "col_transpose", "root_entries", "root_pass2", "root_mask_hdr", "pool_alloc",
           "lprime", "dequeue")
 EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmbe_node_buf_bound_bytes",
            "gmbe_kernel_launch_count",
@@ -50,7 +50,7 @@ class Opts(ctypes.Structure):
                 ("part_count", _u32), ("reserved0", _u32), ("reserved1", _u32),
                 ("out_offsets", _vp), ("out_offsets_cap", _u64), ("out_ids", _vp),
                 ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("phase_cycles", _vp), ("arena_words", _u64),
-                ("slab_words", _u64), ("n_slabs", _u64), ("cuda_stream", _vp)]
+                ("pool_words", _u64), ("queue_cap", _u64), ("cuda_stream", _vp)]
 
 
 class CResult(ctypes.Structure):
@@ -147,7 +147,7 @@ class Graph:
 
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
-                  per_root=False, root_cycles=False, phases=False, debug=0, arena_words=0, slab_words=0, n_slabs=0, stream=None):
+                  per_root=False, root_cycles=False, phases=False, debug=0, arena_words=0, pool_words=0, queue_cap=0, stream=None):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
@@ -155,7 +155,7 @@ class Graph:
         o.no_split = 0 if split else 1
         o.bound_height, o.bound_size, o.warps_per_sm = bound_height, bound_size, warps_per_sm
         o.part_index, o.part_count = part
-        o.arena_words, o.slab_words, o.n_slabs = arena_words, slab_words, n_slabs
+        o.arena_words, o.pool_words, o.queue_cap = arena_words, pool_words, queue_cap
         o.cuda_stream = _stream_ptr(stream)
         o.reserved0 = debug
         bufs = None

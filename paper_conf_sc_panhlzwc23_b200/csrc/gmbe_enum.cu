@@ -42,7 +42,7 @@ struct alignas(128) Line {
   unsigned long long pad[15];
 };
 struct Ctrl {
-  Line root_cursor, q_head, q_tail, f_head, f_tail, pending;
+  Line root_cursor, q_head, q_tail, q_avail, pending, pool_next;
   unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
   unsigned long long out_rec, out_ids;
   unsigned long long phase[16];
@@ -65,12 +65,10 @@ struct Params {
   uint32_t tmax, omax;
   uint32_t* rbuf;     // per-warp R-list stack (only with output)
   uint32_t rbuf_words;
-  uint32_t* slabs;
-  uint64_t slab_words;
-  uint32_t n_slabs;
-  uint32_t* tq;       // task ring (slab ids)
-  uint32_t* fq;       // free-slab ring
-  uint32_t ring_mask;
+  uint32_t* pool;     // task pool: subtasks and shared Γ columns, bump-allocated per call
+  uint64_t pool_words;
+  uint32_t* tq;       // task ring: pool offsets (16-byte units) + 1; 0 = empty slot
+  uint32_t qmask, qcap;
   Ctrl* ctrl;
   unsigned long long* out_offsets;
   uint64_t out_offsets_cap;
@@ -79,7 +77,7 @@ struct Params {
   unsigned long long* per_root;
   unsigned long long* per_root_cycles;
   uint32_t profile;
-  uint32_t debug;  // opts.reserved0 bits (experiments): 1 = no shared column slabs
+  uint32_t debug;  // opts.reserved0 bits (experiments)
 };
 
 struct Acc {
@@ -106,7 +104,7 @@ struct TaskCtx {
   uint32_t* rlist;      // R-list stack (output only)
   const uint32_t* cols; // Γ columns of the root: cols[j*ncw ..] = bitmap of 2-hop vertices adjacent
   uint32_t ncw;         //   to universe vertex j (null: count Γ by binary search)
-  uint32_t colslab;     // slab holding cols when shared with split subtasks (ref-counted), or kNone
+  uint32_t colref;      // pool offset (16-byte units) + 1 of cols when shared with subtasks, else 0
 };
 
 // per-warp memory
@@ -286,81 +284,84 @@ __device__ void warp_sort_keys(unsigned long long* a, uint32_t n, unsigned long 
   warp_bitonic64(a, n);
 }
 
-// ---------------------------------------------------------------- MPMC rings, task slabs (a7)
+// ---------------------------------------------------------------- task pool and queue (a7)
 __device__ __forceinline__ unsigned long long ld_volatile(const unsigned long long* p) {
   return *(volatile const unsigned long long*)p;
 }
-// called by one lane
-__device__ void ring_push(uint32_t* ring, uint32_t mask, unsigned long long* tail, uint32_t x) {
-  const unsigned long long t = atomicAdd(tail, 1ull);
-  uint32_t* slot = ring + (t & mask);
-  while (atomicCAS(slot, GMBE_EMPTY, x) != GMBE_EMPTY) __nanosleep(64);
+// Bump-allocate `words` (multiple of 4) from the task pool; returns the offset in 16-byte units,
+// or kNone when the pool is exhausted (the caller then keeps the work in place).
+__device__ uint32_t pool_alloc(const Params& P, uint64_t words) {
+  unsigned long long off = 0;
+  if (lane_id() == 0) off = atomicAdd(&P.ctrl->pool_next.v, (unsigned long long)words);
+  off = __shfl_sync(GMBE_FULL, off, 0);
+  return off + words <= P.pool_words ? (uint32_t)(off >> 2) : kNone;
 }
-// called by one lane; returns kNone if empty
-__device__ uint32_t ring_pop(uint32_t* ring, uint32_t mask, unsigned long long* head, unsigned long long* tail) {
-  uint32_t backoff = 32;
-  while (true) {
-    const unsigned long long h = ld_volatile(head);
-    const unsigned long long t = ld_volatile(tail);
-    if (h >= t) return kNone;
-    if (atomicCAS(head, h, h + 1) != h) {  // lost the race: back off before retrying
-      __nanosleep(backoff + (clock() & 63));
-      backoff = min(backoff * 2, 4096u);
-    } else {
-      uint32_t* slot = ring + (h & mask);
-      uint32_t x;
-      while ((x = atomicExch(slot, GMBE_EMPTY)) == GMBE_EMPTY) __nanosleep(32);
-      return x;
-    }
+__device__ __forceinline__ uint32_t* pool_ptr(const Params& P, uint32_t off16) { return P.pool + 4ull * off16; }
+// is there room in the task ring (with a margin for concurrent producers)?
+__device__ bool queue_room(const Params& P) {
+  uint32_t ok = 0;
+  if (lane_id() == 0) {
+    const unsigned long long t = ld_volatile(&P.ctrl->q_tail.v), h = ld_volatile(&P.ctrl->q_head.v);
+    ok = t - h + 8192 < P.qcap;
   }
+  return __shfl_sync(GMBE_FULL, ok, 0) != 0;
 }
-__device__ uint32_t slab_alloc(const Params& P) {
-  uint32_t s = kNone;
-  if (lane_id() == 0) s = ring_pop(P.fq, P.ring_mask, &P.ctrl->f_head.v, &P.ctrl->f_tail.v);
-  return __shfl_sync(GMBE_FULL, s, 0);
+// publish a task (one lane): pending += 1, then the slot, then the availability count
+__device__ void queue_push(const Params& P, uint32_t off16) {
+  atomicAdd(&P.ctrl->pending.v, 1ull);
+  const unsigned long long t = atomicAdd(&P.ctrl->q_tail.v, 1ull);
+  uint32_t* slot = P.tq + (t & P.qmask);
+  while (atomicCAS(slot, 0u, off16 + 1) != 0u) __nanosleep(64);
+  atomicAdd(&P.ctrl->q_avail.v, 1ull);
 }
-__device__ void slab_free(const Params& P, uint32_t s) {
-  if (lane_id() == 0) ring_push(P.fq, P.ring_mask, &P.ctrl->f_tail.v, s);
+// take a task (one lane): reserve through the availability count (fetch-add, no CAS storms), then
+// claim the next ticket and wait for its slot.  Returns kNone if nothing is available.
+__device__ uint32_t queue_pop(const Params& P) {
+  if ((long long)ld_volatile(&P.ctrl->q_avail.v) <= 0) return kNone;
+  if ((long long)atomicAdd(&P.ctrl->q_avail.v, ~0ull) <= 0) {
+    atomicAdd(&P.ctrl->q_avail.v, 1ull);
+    return kNone;
+  }
+  const unsigned long long h = atomicAdd(&P.ctrl->q_head.v, 1ull);
+  uint32_t* slot = P.tq + (h & P.qmask);
+  uint32_t x;
+  while ((x = atomicExch(slot, 0u)) == 0u) __nanosleep(32);
+  return x - 1;
 }
-// drop one reference to a shared column slab; the last holder frees it
-__device__ void colslab_release(const Params& P, uint32_t cs) {
-  if (cs == kNone) return;
-  uint32_t last = 0;
-  if (lane_id() == 0) last = atomicSub(P.slabs + (uint64_t)cs * P.slab_words, 1u) == 1u;
-  last = __shfl_sync(GMBE_FULL, last, 0);
-  if (last) slab_free(P, cs);
-}
-// task slab layout: [0]=W [1]=map length [2]=root rank [3]=R length [4]=node offset
-//                   [5]=column slab (or kNone) [6]=column words [7] pad | map | R list | node record
-// column slab layout: [0]=reference count [1..7] pad | columns
-__device__ __forceinline__ uint32_t slab_node_off(uint32_t lmap, uint32_t rlen) { return kHdr + r4(lmap) + r4(rlen); }
-// Publish the child node already written at slab + node_off as a self-contained subtask (Alg 4 L25).
-__device__ void slab_publish(const Params& P, uint32_t slab, const TaskCtx& T, uint32_t lmap, uint32_t rlen,
-                             uint32_t node_off, Acc& A) {
+// task record: [0]=W [1]=map length [2]=root rank [3]=R length [4]=node offset [5]=colref
+//              [6]=column words [7] pad | map | R list | node record
+__device__ __forceinline__ uint32_t task_node_off(uint32_t lmap, uint32_t rlen) { return kHdr + r4(lmap) + r4(rlen); }
+// Copy the node record `rec` (words) into a new self-contained subtask and publish it (Alg 4 L25).
+// Returns false (nothing published) if the pool or the queue is full.
+__device__ bool task_publish(const Params& P, const TaskCtx& T, uint32_t lmap, uint32_t rlen, const uint32_t* rec,
+                             uint32_t words, Acc& A) {
   const uint32_t lane = lane_id();
-  uint32_t* s = P.slabs + (uint64_t)slab * P.slab_words;
+  if (!queue_room(P)) return false;
+  const uint32_t node_off = task_node_off(lmap, T.rlist ? rlen : 0);
+  const uint32_t off16 = pool_alloc(P, r4(node_off + words));
+  if (off16 == kNone) return false;
+  uint32_t* s = pool_ptr(P, off16);
   for (uint32_t j = lane; j < lmap; j += 32) s[kHdr + j] = T.map[j];
   if (T.rlist)
     for (uint32_t j = lane; j < rlen; j += 32) s[kHdr + r4(lmap) + j] = T.rlist[j];
+  for (uint32_t j = lane; j < words; j += 32) s[node_off + j] = rec[j];
+  __syncwarp();
   if (lane == 0) {
     s[0] = T.W;
     s[1] = lmap;
     s[2] = T.root;
     s[3] = T.rlist ? rlen : 0;
     s[4] = node_off;
-    s[5] = T.colslab;
+    s[5] = T.colref;
     s[6] = T.ncw;
     s[node_off + 3] = 0;      // next candidate
     s[node_off + 4] = kNone;  // no parent: top of its task
-    if (T.colslab != kNone) atomicAdd(P.slabs + (uint64_t)T.colslab * P.slab_words, 1u);
   }
   A.tasks++;
-  __threadfence();  // release the slab contents before it becomes visible in the queue
+  __threadfence();  // release the task before it becomes visible in the queue
   __syncwarp();
-  if (lane == 0) {
-    atomicAdd(&P.ctrl->pending.v, 1ull);
-    ring_push(P.tq, P.ring_mask, &P.ctrl->q_tail.v, slab);
-  }
+  if (lane == 0) queue_push(P, off16);
+  return true;
 }
 
 // ---------------------------------------------------------------- emission (a8)
@@ -705,20 +706,9 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     if (r == 2 && split_mode && cur == top) {
       // Alg 4 L25: hand the child to the task queue as a self-contained subtask
       PH_START(A);
-      const uint32_t words = rec_words(T, ch);
-      const uint32_t rlen = T.rlist ? ch[5] : 0;
-      const uint32_t node_off = slab_node_off(lmap, rlen);
-      uint32_t slab = kNone;
-      if (node_off + words <= P.slab_words) slab = slab_alloc(P);
-      PH_STOP(A, 13);
-      if (slab != kNone) {
-        uint32_t* dst = P.slabs + (uint64_t)slab * P.slab_words + node_off;
-        for (uint32_t j = lane; j < words; j += 32) dst[j] = ch[j];
-        __syncwarp();
-        slab_publish(P, slab, T, lmap, rlen, node_off, A);
-        PH_STOP(A, 7);
-        continue;
-      }
+      const bool done = task_publish(P, T, lmap, T.rlist ? ch[5] : 0, ch, rec_words(T, ch), A);
+      PH_STOP(A, 7);
+      if (done) continue;
     }
     if (r == 2) {  // push (Alg 2 L16)
       if (lane == 0) {
@@ -922,24 +912,21 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       Tc.rlist = M.rbuf;
       Tc.cols = want_cols ? cols : nullptr;
       Tc.ncw = ncw;
-      Tc.colslab = kNone;
+      Tc.colref = 0;
       PH_STOP(A, 12);
-      if (!(P.debug & 1) && want_cols && heavy(P, l, nC) && kHdr + (uint64_t)l * ncw <= P.slab_words) {
-        // the root will be split: share its columns with the subtasks through a ref-counted slab
-        const uint32_t cs = slab_alloc(P);
-        if (cs != kNone) {
-          uint32_t* csp = P.slabs + (uint64_t)cs * P.slab_words;
-          for (uint64_t j = lane; j < (uint64_t)l * ncw; j += 32) csp[kHdr + j] = cols[j];
-          if (lane == 0) csp[0] = 1;
-          __threadfence();
+      if (want_cols && heavy(P, l, nC)) {
+        // the root will be split: share its Γ columns with the subtasks through the task pool
+        const uint32_t co = pool_alloc(P, r4(l * ncw));
+        if (co != kNone) {
+          uint32_t* cp = pool_ptr(P, co);
+          for (uint64_t j = lane; j < (uint64_t)l * ncw; j += 32) cp[j] = cols[j];
           __syncwarp();
-          Tc.cols = csp + kHdr;
-          Tc.colslab = cs;
+          Tc.cols = cp;
+          Tc.colref = co + 1;
         }
       }
       PH_STOP(A, 3);
       dispatch_task(P, Tc, rec, align4(rec + rec_need), M.dyn_end, l, A, M.sm_sort);
-      colslab_release(P, Tc.colslab);
     }
   }
   // leave the table clean for the next root
@@ -971,12 +958,12 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
   while (true) {
     // 1. split subtasks first (Alg 4 L3-4)
     uint32_t task = kNone;
-    if (lane == 0) task = ring_pop(P.tq, P.ring_mask, &P.ctrl->q_head.v, &P.ctrl->q_tail.v);
+    if (lane == 0) task = queue_pop(P);
     task = __shfl_sync(GMBE_FULL, task, 0);
     if (task != kNone) {
       PH_START(A);
-      __threadfence();  // acquire: the slab was written on another SM
-      uint32_t* s = P.slabs + (uint64_t)task * P.slab_words;
+      __threadfence();  // acquire: the task was written on another SM
+      uint32_t* s = pool_ptr(P, task);
       TaskCtx Tc;
       Tc.W = s[0];
       const uint32_t lmap = s[1];
@@ -986,9 +973,9 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       Tc.E = r4(Tc.W + 2);
       Tc.map = s + kHdr;
       Tc.rlist = M.rbuf;
-      Tc.colslab = s[5];
+      Tc.colref = s[5];
       Tc.ncw = s[6];
-      Tc.cols = Tc.colslab != kNone ? P.slabs + (uint64_t)Tc.colslab * P.slab_words + kHdr : nullptr;
+      Tc.cols = Tc.colref ? pool_ptr(P, Tc.colref - 1) : nullptr;
       if (M.rbuf)
         for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
       __syncwarp();
@@ -998,8 +985,6 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       if (P.per_root_cycles && lane == 0)
         atomicAdd(P.per_root_cycles + Tc.root, (unsigned long long)(clock64() - c0));
       __syncwarp();
-      colslab_release(P, Tc.colslab);
-      slab_free(P, task);
       if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
       idle = 0;
       continue;
@@ -1049,13 +1034,6 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
   }
 }
 
-__global__ void k_init_rings(uint32_t* tq, uint32_t* fq, uint32_t cap, uint32_t n_slabs) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < cap; i += gridDim.x * blockDim.x) {
-    tq[i] = GMBE_EMPTY;
-    fq[i] = i < n_slabs ? i : GMBE_EMPTY;
-  }
-}
-
 // ---------------------------------------------------------------- host side
 struct Workspace {
   int device = -1;
@@ -1063,8 +1041,8 @@ struct Workspace {
   size_t arena_bytes = 0;
   uint64_t layout[4] = {0, 0, 0, 0};  // tmax, omax, arena_words, nwarps of the clean tables
   bool clean = false;
-  void* slabs = nullptr;
-  size_t slab_bytes = 0;
+  void* pool = nullptr;
+  size_t pool_bytes = 0;
   void* rings = nullptr;
   size_t ring_bytes = 0;
   void* rbuf = nullptr;
@@ -1125,7 +1103,7 @@ extern "C" void gmbe_release_workspace(const gmbe_graph* G) {
       i++;
       continue;
     }
-    for (void* p : {w->arena, w->slabs, w->rings, w->rbuf, w->ctrl, w->per_root, w->per_root_cyc})
+    for (void* p : {w->arena, w->pool, w->rings, w->rbuf, w->ctrl, w->per_root, w->per_root_cyc})
       if (p) cudaFree(p);
     delete w;
     g_ws_idle.erase(g_ws_idle.begin() + i);
@@ -1187,12 +1165,17 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
     dyn = want < cap ? want : cap;
   }
   const uint64_t arena_words = (fixed + dyn + 3) & ~3ull;
-  uint64_t slab_words = o.slab_words ? o.slab_words : (1u << 16);
-  slab_words = (slab_words + 3) & ~3ull;
-  uint64_t n_slabs = o.n_slabs ? o.n_slabs : 8192;
-  if (n_slabs > (1u << 24)) n_slabs = 1u << 24;
+  uint64_t pool_words = o.pool_words;
+  if (!pool_words) {  // task pool: subtasks + shared columns, never reused within a call
+    size_t fr = 0, tot = 0;
+    GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
+    pool_words = std::min<uint64_t>(1ull << 30, (uint64_t)(fr * 0.2) / 4);
+  }
+  pool_words = (pool_words + 3) & ~3ull;
   uint32_t cap = 1;
-  while (cap < n_slabs + 64) cap <<= 1;
+  const uint64_t want_cap = o.queue_cap ? o.queue_cap : (1u << 20);
+  while (cap < want_cap && cap < (1u << 30)) cap <<= 1;
+  if (cap < 16384) cap = 16384;  // > the producers' admission margin
   const bool want_out = o.out_ids != nullptr;
   const uint32_t rbuf_words = want_out ? (uint32_t)(wb + 64) : 0;
 
@@ -1207,8 +1190,8 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
       W.clean = true;
     }
   }
-  GMBE_CUDA_TRY(ensure(&W.slabs, &W.slab_bytes, n_slabs * slab_words * 4));
-  GMBE_CUDA_TRY(ensure(&W.rings, &W.ring_bytes, (size_t)cap * 2 * 4));
+  GMBE_CUDA_TRY(ensure(&W.pool, &W.pool_bytes, pool_words * 4));
+  GMBE_CUDA_TRY(ensure(&W.rings, &W.ring_bytes, (size_t)cap * 4));
   if (want_out) GMBE_CUDA_TRY(ensure(&W.rbuf, &W.rbuf_bytes, nwarps * rbuf_words * 4));
   GMBE_CUDA_TRY(ensure(&W.ctrl, &W.ctrl_bytes, sizeof(Ctrl)));
   if (o.per_root_count) GMBE_CUDA_TRY(ensure(&W.per_root, &W.per_root_bytes, (size_t)(g.n_v + 1) * 8));
@@ -1231,12 +1214,11 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.omax = (uint32_t)omax;
   P.rbuf = want_out ? (uint32_t*)W.rbuf : nullptr;
   P.rbuf_words = rbuf_words;
-  P.slabs = (uint32_t*)W.slabs;
-  P.slab_words = slab_words;
-  P.n_slabs = (uint32_t)n_slabs;
+  P.pool = (uint32_t*)W.pool;
+  P.pool_words = pool_words;
   P.tq = (uint32_t*)W.rings;
-  P.fq = (uint32_t*)W.rings + cap;
-  P.ring_mask = cap - 1;
+  P.qmask = cap - 1;
+  P.qcap = cap;
   P.ctrl = (Ctrl*)W.ctrl;
   P.out_offsets = (unsigned long long*)o.out_offsets;
   P.out_offsets_cap = want_out ? o.out_offsets_cap : 0;
@@ -1248,10 +1230,8 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.debug = o.reserved0;
 
   Ctrl hc{};
-  hc.f_tail.v = n_slabs;
   GMBE_CUDA_TRY(cudaMemcpyAsync(W.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
-  k_init_rings<<<(cap + 255) / 256 < 1024 ? (cap + 255) / 256 : 1024, 256, 0, s>>>(P.tq, P.fq, cap, (uint32_t)n_slabs);
-  gmbe_note_launch();
+  GMBE_CUDA_TRY(cudaMemsetAsync(W.rings, 0, (size_t)cap * 4, s));
   if (P.per_root) GMBE_CUDA_TRY(cudaMemsetAsync(W.per_root, 0, (size_t)(g.n_v + 1) * 8, s));
   if (P.per_root_cycles) GMBE_CUDA_TRY(cudaMemsetAsync(W.per_root_cyc, 0, (size_t)(g.n_v + 1) * 8, s));
   GMBE_CUDA_TRY(cudaGetLastError());
@@ -1298,7 +1278,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   if (hc.error) {
     W.clean = false;
     return gmbe_set_error(GMBE_EINTERNAL,
-                          "gmbe_enumerate: per-warp workspace exceeded; raise opts.arena_words / slab_words");
+                          "gmbe_enumerate: per-warp workspace exceeded; raise opts.arena_words");
   }
   return GMBE_OK;
 }

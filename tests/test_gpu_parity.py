@@ -162,17 +162,17 @@ def test_split_and_schedule_invariance(gmbe, dense_case):
     g = gmbe.load(nu, nv, e)
     try:
         variants = [dict(), dict(split=False), dict(bound_height=1, bound_size=1),
-                    dict(bound_height=1, bound_size=1, n_slabs=1),
-                    dict(bound_height=1, bound_size=1, n_slabs=3, slab_words=4096),
+                    dict(bound_height=1, bound_size=1, pool_words=64),
+                    dict(bound_height=1, bound_size=1, pool_words=4096),
                     dict(warps_per_sm=8), dict(warps_per_sm=64),
-                    dict(bound_height=2, bound_size=8, n_slabs=2), dict(arena_words=4096)]
+                    dict(bound_height=2, bound_size=8, pool_words=2048), dict(arena_words=4096)]
         for kw in variants:
             r = g.enumerate(**kw)
             _same(r, o)
             assert r.algo_bytes_cand == o.algo_bytes_cand, kw
-        for nsl in (0, 2):
-            r = g.enumerate(bound_height=1, bound_size=1, records=True, n_slabs=nsl)
-            assert r.tasks > 0 and r.splits > 0
+        for pw in (0, 1024):
+            r = g.enumerate(bound_height=1, bound_size=1, records=True, pool_words=pw)
+            assert r.splits > 0 and (r.tasks > 0 or pw)
             assert r.bicliques == sorted(o.bicliques)
     finally:
         g.free()
