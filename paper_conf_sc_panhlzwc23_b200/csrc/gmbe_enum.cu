@@ -102,9 +102,15 @@ struct TaskCtx {
   uint32_t W, W4, E;    // words per row, padded L-mask words, entry stride
   uint32_t root;        // rank of the root vertex
   uint32_t* rlist;      // R-list stack (output only)
-  const uint32_t* cols; // Γ columns of the root: cols[j*ncw ..] = bitmap of 2-hop vertices adjacent
-  uint32_t ncw;         //   to universe vertex j (null: count Γ by binary search)
-  uint32_t colref;      // pool offset (16-byte units) + 1 of cols when shared with subtasks, else 0
+  // Γ index of the root (maximality count without binary searches), one of:
+  //   gx  (universe <= 64 bits): [nx, l, -, -] | xrow u64[nx] (row of each 2-hop vertex x over the
+  //        universe) | coff u32[l+1] | cx u32[] (2-hop indices adjacent to universe vertex j)
+  //   cols (larger universes): cols[j*ncw ..] = bitmap of the 2-hop vertices adjacent to vertex j
+  // or neither (count Γ by binary search over the adjacency lists).
+  const uint32_t* gx;
+  const uint32_t* cols;
+  uint32_t ncw;
+  uint32_t auxref;      // pool offset (16-byte units) + 1 of gx / cols when shared with subtasks, else 0
 };
 
 // per-warp memory
@@ -328,8 +334,8 @@ __device__ uint32_t queue_pop(const Params& P) {
   while ((x = atomicExch(slot, 0u)) == 0u) __nanosleep(32);
   return x - 1;
 }
-// task record: [0]=W [1]=map length [2]=root rank [3]=R length [4]=node offset [5]=colref
-//              [6]=column words [7] pad | map | R list | node record
+// task record: [0]=W [1]=map length [2]=root rank [3]=R length [4]=node offset [5]=auxref
+//              [6]=column words [7]=aux kind (0 none, 1 cols, 2 gx) | map | R list | node record
 __device__ __forceinline__ uint32_t task_node_off(uint32_t lmap, uint32_t rlen) { return kHdr + r4(lmap) + r4(rlen); }
 // Copy the node record `rec` (words) into a new self-contained subtask and publish it (Alg 4 L25).
 // Returns false (nothing published) if the pool or the queue is full.
@@ -352,8 +358,9 @@ __device__ bool task_publish(const Params& P, const TaskCtx& T, uint32_t lmap, u
     s[2] = T.root;
     s[3] = T.rlist ? rlen : 0;
     s[4] = node_off;
-    s[5] = T.colref;
+    s[5] = T.auxref;
     s[6] = T.ncw;
+    s[7] = T.auxref ? (T.gx ? 2u : 1u) : 0u;
     s[node_off + 3] = 0;      // next candidate
     s[node_off + 4] = kNone;  // no parent: top of its task
   }
@@ -524,6 +531,36 @@ __device__ bool gamma_cols_is_r(const TaskCtx& T, const uint32_t* lmask, uint32_
   return count == need;
 }
 
+// Alg 2 L14 with the root's Γ index gx (universe <= 64 bits, L' = lm): Γ(L') ⊆ {v_s} ∪ {x adjacent to
+// u*} for the lowest-degree u* ∈ L'; count the x whose row covers L'.  |Γ(L')| <= deg(u*), so
+// deg(u*) == |R'| proves maximality at once.
+__device__ bool gamma_gx_is_r(const uint32_t* gx, unsigned long long lm, uint32_t rlen) {
+  const uint32_t lane = lane_id();
+  const uint32_t nx = gx[0], l = gx[1];
+  const unsigned long long* xrow = (const unsigned long long*)(gx + 4);
+  const uint32_t* coff = gx + 4 + 2 * nx;
+  const uint32_t* cx = coff + r4(l + 1);
+  // j* = argmin over members of |list_j| (= deg(u_j) - 1)
+  uint32_t key = 0xffffffffu;
+  for (uint32_t j = lane; j < l; j += 32)
+    if ((lm >> j) & 1ull) key = min(key, ((coff[j + 1] - coff[j]) << 7) | j);
+  key = __reduce_min_sync(GMBE_FULL, key);
+  const uint32_t js = key & 127u, len = key >> 7;
+  if (len + 1 == rlen) return true;
+  uint32_t count = 1;  // v_s
+  const uint32_t* lst = cx + coff[js];
+  for (uint32_t b = 0; b < len; b += 32) {
+    bool full = false;
+    if (b + lane < len) {
+      const unsigned long long row = xrow[lst[b + lane]];
+      full = (row & lm) == lm;
+    }
+    count += __popc(__ballot_sync(GMBE_FULL, full));
+    if (count > rlen) return false;
+  }
+  return count == rlen;
+}
+
 // ---------------------------------------------------------------- child generation (a4, a5)
 // Generate the child of node `par` via its candidate i into `ch` (Alg 2 L6-16).  The parent's later
 // candidates are compacted in place (Thm 4.1 prunes removed), so par[0] shrinks.
@@ -626,6 +663,9 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
     while (!lpm[w]) w++;
     const uint32_t u = T.map[w * 32 + __ffs(lpm[w]) - 1];
     maximal = P.g.off_u[u + 1] - P.g.off_u[u] == rlen;
+  } else if (T.gx) {
+    const unsigned long long lm = W == 1 ? lpm[0] : ((unsigned long long)lpm[1] << 32) | lpm[0];
+    maximal = gamma_gx_is_r(T.gx, lm, rlen);
   } else if (T.cols) {
     maximal = gamma_cols_is_r(T, lpm, W, rlen);
   } else {
@@ -800,11 +840,16 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
   }
   skip = __any_sync(GMBE_FULL, skip);
   PH_STOP(A, 1);
-  // Γ columns over the 2-hop set X (= the occupied table slots; x = position in occ)
+  // Γ index over the 2-hop set X (= the occupied table slots; x = position in occ): gx for
+  // universes <= 64 bits, columns otherwise (see TaskCtx)
   const uint32_t ncw = (nocc + 31) / 32;
-  uint32_t* cols = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
-  const bool want_cols = !skip && nC > 0 && (uint64_t)l * ncw <= P.col_budget;
-  uint32_t* rec = align4(cols + (want_cols ? (size_t)l * ncw : 0));
+  uint32_t* aux = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
+  const uint64_t aux_words = small ? 4ull + 2ull * nocc + r4(l + 1) + (wedges - l) : (uint64_t)l * ncw;
+  const bool want_aux = !skip && nC > 0 && aux_words <= P.col_budget;
+  const bool want_cols = want_aux && !small;
+  uint32_t* cols = aux;
+  uint32_t* gx = aux;
+  uint32_t* rec = align4(aux + (want_aux ? aux_words : 0));
   const uint64_t rec_need = kHdr + W4 + (uint64_t)nC * E;
   if (sort_fits && !skip && fits(P, rec + rec_need + 64, M.dyn_end)) {
     A.roots_run++;
@@ -821,21 +866,49 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       if (P.out_ids) write_record(P, nullptr, 0, nullptr, Lr, l, M.rbuf, nR + 1);
     }
     PH_STOP(A, 8);
-    if (want_cols && small) {
-      // transpose the table rows (<= 64 bits) into columns with ballots
+    if (want_aux && small) {
+      // gx: rows of the 2-hop vertices, and per universe vertex u_j the list of its 2-hop
+      // neighbours (|list_j| = deg(u_j) - 1: every neighbour but v_s lies in X)
+      unsigned long long* xrow = (unsigned long long*)(gx + 4);
+      uint32_t* coff = gx + 4 + 2 * nocc;
+      uint32_t* cx = coff + r4(l + 1);
+      if (lane == 0) {
+        gx[0] = nocc;
+        gx[1] = l;
+      }
+      for (uint32_t x = lane; x < nocc; x += 32) xrow[x] = __ldcg(vals + M.occ[x]);
+      uint32_t carry = 0, cur0 = 0, cur1 = 0;
+      for (uint32_t h = 0; h < 2; h++) {
+        const uint32_t j = h * 32 + lane;
+        const uint32_t c = j < l ? g.off_u[Lr[j] + 1] - g.off_u[Lr[j]] - 1 : 0;
+        uint32_t inc = c;
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t t = __shfl_up_sync(GMBE_FULL, inc, o);
+          if (lane >= (uint32_t)o) inc += t;
+        }
+        const uint32_t ex = carry + inc - c;
+        if (j <= l) coff[j] = ex;
+        if (h == 0) cur0 = ex;
+        else cur1 = ex;
+        carry += __shfl_sync(GMBE_FULL, inc, 31);
+      }
+      if (lane == 0 && l == 64) coff[64] = carry;
+      __syncwarp();
       for (uint32_t b = 0; b < nocc; b += 32) {
         const uint32_t x = b + lane;
-        const unsigned long long row = x < nocc ? __ldcg(vals + M.occ[x]) : 0ull;
-        uint32_t mine0 = 0, mine1 = 0;
+        const unsigned long long row = x < nocc ? xrow[x] : 0ull;
         for (uint32_t j = 0; j < l; j++) {
-          const uint32_t bal = __ballot_sync(GMBE_FULL, (row >> j) & 1ull);
-          if (lane == (j & 31)) {
-            if (j < 32) mine0 = bal;
-            else mine1 = bal;
+          const bool bit = (row >> j) & 1ull;
+          const uint32_t bal = __ballot_sync(GMBE_FULL, bit);
+          if (bal) {
+            const uint32_t base = __shfl_sync(GMBE_FULL, j < 32 ? cur0 : cur1, j & 31);
+            if (bit) cx[base + __popc(bal & lanemask_lt())] = x;
+            if (lane == (j & 31)) {
+              if (j < 32) cur0 += __popc(bal);
+              else cur1 += __popc(bal);
+            }
           }
         }
-        if (lane < l) cols[(size_t)lane * ncw + (b >> 5)] = mine0;
-        if (lane + 32 < l) cols[(size_t)(lane + 32) * ncw + (b >> 5)] = mine1;
       }
       __syncwarp();
     }
@@ -911,18 +984,20 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       Tc.root = r;
       Tc.rlist = M.rbuf;
       Tc.cols = want_cols ? cols : nullptr;
+      Tc.gx = want_aux && small ? gx : nullptr;
       Tc.ncw = ncw;
-      Tc.colref = 0;
+      Tc.auxref = 0;
       PH_STOP(A, 12);
-      if (want_cols && heavy(P, l, nC)) {
-        // the root will be split: share its Γ columns with the subtasks through the task pool
-        const uint32_t co = pool_alloc(P, r4(l * ncw));
+      if (want_aux && heavy(P, l, nC)) {
+        // the root will be split: share its Γ index with the subtasks through the task pool
+        const uint32_t co = pool_alloc(P, r4((uint32_t)aux_words));
         if (co != kNone) {
           uint32_t* cp = pool_ptr(P, co);
-          for (uint64_t j = lane; j < (uint64_t)l * ncw; j += 32) cp[j] = cols[j];
+          for (uint64_t j = lane; j < aux_words; j += 32) cp[j] = aux[j];
           __syncwarp();
-          Tc.cols = cp;
-          Tc.colref = co + 1;
+          if (small) Tc.gx = cp;
+          else Tc.cols = cp;
+          Tc.auxref = co + 1;
         }
       }
       PH_STOP(A, 3);
@@ -973,9 +1048,10 @@ __global__ void __launch_bounds__(256) k_enum(const Params P) {
       Tc.E = r4(Tc.W + 2);
       Tc.map = s + kHdr;
       Tc.rlist = M.rbuf;
-      Tc.colref = s[5];
+      Tc.auxref = s[5];
       Tc.ncw = s[6];
-      Tc.cols = Tc.colref ? pool_ptr(P, Tc.colref - 1) : nullptr;
+      Tc.cols = s[7] == 1 ? pool_ptr(P, Tc.auxref - 1) : nullptr;
+      Tc.gx = s[7] == 2 ? pool_ptr(P, Tc.auxref - 1) : nullptr;
       if (M.rbuf)
         for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
       __syncwarp();
