@@ -111,6 +111,10 @@ struct TaskCtx {
   const uint32_t* cols;
   uint32_t ncw;
   uint32_t auxref;      // pool offset (16-byte units) + 1 of gx / cols when shared with subtasks, else 0
+  // lane-resident copies for universes <= 64 bits (universe vertices lane and lane + 32), filled by
+  // small_task_init: Γ-list offsets / lengths and the checksum hashes of the universe vertices
+  uint32_t go0, go1, gl0, gl1;
+  unsigned long long hu0, hu1;
 };
 
 // per-warp memory
@@ -134,6 +138,13 @@ __device__ __forceinline__ uint32_t warp_sum(uint32_t x) { return __reduce_add_s
 __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
   for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(GMBE_FULL, x, o);
   return x;
+}
+// 64-bit warp sum with three 32-bit REDUX ops (21/21/22-bit limbs cannot overflow over 32 lanes)
+__device__ __forceinline__ unsigned long long warp_sum64r(unsigned long long x) {
+  const uint32_t a = __reduce_add_sync(GMBE_FULL, (uint32_t)(x & 0x1fffffull));
+  const uint32_t b = __reduce_add_sync(GMBE_FULL, (uint32_t)((x >> 21) & 0x1fffffull));
+  const uint32_t c = __reduce_add_sync(GMBE_FULL, (uint32_t)(x >> 42));
+  return (unsigned long long)a + ((unsigned long long)b << 21) + ((unsigned long long)c << 42);
 }
 template <int LPE>
 __device__ __forceinline__ uint32_t group_sum(uint32_t x) {
@@ -708,6 +719,155 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   return 2;
 }
 
+// ---------------------------------------------------------------- small universes (<= 64 bits)
+// Per-task lane-resident data for W <= 2 (see TaskCtx).
+__device__ void small_task_init(const Params& P, TaskCtx& T, uint32_t lmap) {
+  const uint32_t lane = lane_id();
+  T.go0 = T.go1 = T.gl0 = T.gl1 = 0;
+  T.hu0 = lane < lmap ? gmbe_hid(T.map[lane], P.hu_side) : 0ull;
+  T.hu1 = lane + 32 < lmap ? gmbe_hid(T.map[lane + 32], P.hu_side) : 0ull;
+  if (T.gx) {
+    const uint32_t* coff = T.gx + 4 + 2 * T.gx[0];
+    const uint32_t l = T.gx[1];
+    if (lane < l) {
+      T.go0 = coff[lane];
+      T.gl0 = coff[lane + 1] - T.go0;
+    }
+    if (lane + 32 < l) {
+      T.go1 = coff[lane + 32];
+      T.gl1 = coff[lane + 33] - T.go1;
+    }
+  }
+}
+
+// maximality with gx and lane-resident list offsets (see gamma_gx_is_r)
+__device__ __forceinline__ bool gamma_gx_small(const TaskCtx& T, unsigned long long lm, uint32_t rlen) {
+  const uint32_t lane = lane_id();
+  uint32_t key = 0xffffffffu;
+  if ((lm >> lane) & 1ull) key = (T.gl0 << 7) | lane;
+  if ((lm >> (lane + 32)) & 1ull) key = min(key, (T.gl1 << 7) | (lane + 32));
+  key = __reduce_min_sync(GMBE_FULL, key);
+  const uint32_t js = key & 127u, len = key >> 7;
+  if (len + 1 == rlen) return true;  // |Γ(L')| <= deg(u*) = len + 1
+  const uint32_t off = __shfl_sync(GMBE_FULL, js < 32 ? T.go0 : T.go1, js & 31);
+  const uint32_t nx = T.gx[0];
+  const unsigned long long* xrow = (const unsigned long long*)(T.gx + 4);
+  const uint32_t* lst = T.gx + 4 + 2 * nx + r4(T.gx[1] + 1) + off;
+  uint32_t count = 1;  // v_s
+  for (uint32_t b = 0; b < len; b += 32) {
+    bool full = false;
+    if (b + lane < len) full = (xrow[lst[b + lane]] & lm) == lm;
+    count += __popc(__ballot_sync(GMBE_FULL, full));
+    if (count > rlen) return false;
+  }
+  return count == rlen;
+}
+
+// gen_child for W <= 2: one lane per candidate entry, loaded as one 16-byte vector
+// ({row, id, k, -} for W = 1, {row_lo, row_hi, id, k} for W = 2); L' and rows as 64-bit masks.
+__device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par, uint32_t i, uint32_t* ch, Acc& A,
+                               unsigned long long* smem) {
+  const uint32_t lane = lane_id();
+  const bool w2 = T.W == 2;
+  const uint32_t nC = par[0];
+  uint4* pent = (uint4*)(par + kHdr + 4);
+  uint4* cent = (uint4*)(ch + kHdr + 4);
+  PH_START(A);
+  const uint4 vr = pent[i];
+  const unsigned long long vrow = w2 ? (((unsigned long long)vr.y << 32) | vr.x) : vr.x;
+  const uint32_t vid = w2 ? vr.z : vr.y;
+  const unsigned long long lpar = ((unsigned long long)par[kHdr + 1] << 32) | par[kHdr];
+  const unsigned long long lm = lpar & vrow;  // L' = L_p ∩ N(v')   (Alg 2 L8)
+  const uint32_t lc = __popcll(lm);
+  if (lane == 0) {
+    ch[kHdr] = (uint32_t)lm;
+    ch[kHdr + 1] = (uint32_t)(lm >> 32);
+  }
+  PH_STOP(A, 14);
+  // later candidates: k' (Alg 2 L9-13), Thm 4.1 pruning with in-place compaction, R', C'
+  uint32_t nCc = 0, nsurv = 0, r_abs = 0;
+  unsigned long long sr_abs = 0, later_k = 0;
+  const uint32_t rl_base = par[5] + 1;
+  for (uint32_t base = i + 1; base < nC; base += 32) {
+    const uint32_t j = base + lane;
+    const bool in = j < nC;
+    uint4 x = make_uint4(0, 0, 0, 0);
+    if (in) x = pent[j];
+    const unsigned long long row = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
+    const uint32_t id = w2 ? x.z : x.y, kp = w2 ? x.w : x.z;
+    const unsigned long long xr = row & lm;
+    const uint32_t cnt = __popcll(xr);
+    const bool pruned = in && P.prune && cnt == kp;
+    const bool surv = in && !pruned;
+    const bool absorb = in && cnt == lc;
+    const bool cand = in && cnt > 0 && cnt < lc;
+    if (in) later_k += kp;
+    if (absorb) sr_abs += P.g.hv[id];
+    const uint32_t ba = __ballot_sync(GMBE_FULL, absorb);
+    if (T.rlist && absorb) T.rlist[rl_base + r_abs + __popc(ba & lanemask_lt())] = id;
+    r_abs += __popc(ba);
+    const uint32_t bc = __ballot_sync(GMBE_FULL, cand);
+    if (cand)
+      cent[nCc + __popc(bc & lanemask_lt())] =
+          w2 ? make_uint4((uint32_t)xr, (uint32_t)(xr >> 32), id, cnt) : make_uint4((uint32_t)xr, id, cnt, 0);
+    nCc += __popc(bc);
+    const uint32_t bs = __ballot_sync(GMBE_FULL, surv);
+    const uint32_t spos = i + 1 + nsurv + __popc(bs & lanemask_lt());
+    nsurv += __popc(bs);
+    __syncwarp();
+    if (surv && spos != j) pent[spos] = x;
+    __syncwarp();
+  }
+  if (lane == 0) par[0] = i + 1 + nsurv;
+  A.nodes++;
+  A.abytes += 4ull * (lc + warp_sum64r(later_k));
+  const uint32_t rlen = par[5] + 1 + r_abs;
+  PH_STOP(A, 4);
+  bool maximal;
+  if (lc == 1) {  // Γ({u}) = N(u)
+    const uint32_t j = __ffsll(lm) - 1;
+    const uint32_t u = T.map[j];
+    maximal = P.g.off_u[u + 1] - P.g.off_u[u] == rlen;
+  } else if (T.gx) {
+    maximal = gamma_gx_small(T, lm, rlen);
+  } else {
+    __syncwarp();
+    maximal = gamma_is_r(P, ch + kHdr, T.W, T.map, lc, rlen,
+                         (unsigned long long*)align4((uint32_t*)(cent + nCc)), smem);
+  }
+  PH_STOP(A, 5);
+  if (!maximal) {
+    A.nonmax++;
+    return 0;
+  }
+  // Output(L', R') (Alg 2 L15)
+  const unsigned long long par_sr = ((unsigned long long)par[7] << 32) | par[6];
+  const unsigned long long sl =
+      warp_sum64r(((lm >> lane) & 1ull ? T.hu0 : 0ull) + ((lm >> (lane + 32)) & 1ull ? T.hu1 : 0ull));
+  const unsigned long long sr = par_sr + P.g.hv[vid] + warp_sum64r(sr_abs);
+  A.count++;
+  A.checksum += pair_hash(P, sl, sr);
+  if (P.per_root && lane == 0) atomicAdd(P.per_root + T.root, 1ull);
+  if (T.rlist) {
+    if (lane == 0) T.rlist[par[5]] = vid;
+    __syncwarp();
+    if (P.out_ids) write_record(P, ch + kHdr, T.W, T.map, nullptr, lc, T.rlist, rlen);
+  }
+  PH_STOP(A, 6);
+  if (nCc == 0) return 1;
+  if (lane == 0) {
+    ch[0] = nCc;
+    ch[1] = 0;
+    ch[2] = lc;
+    ch[3] = 0;
+    ch[5] = rlen;
+    ch[6] = (uint32_t)sr;
+    ch[7] = (uint32_t)(sr >> 32);
+  }
+  __syncwarp();
+  return 2;
+}
+
 __device__ __forceinline__ uint32_t rec_words(const TaskCtx& T, const uint32_t* rec) {
   return kHdr + T.W4 + rec[0] * T.E;
 }
@@ -742,7 +902,9 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     const uint64_t need = kHdr + T.W4 + (uint64_t)(cur[0] - i - 1) * T.E + 4ull * 32 * T.W + 16;
     if (!fits(P, sp + need, stack_hi)) return;
     uint32_t* ch = sp;  // children are generated on this warp's stack; only a published one is copied
-    const int r = gen_child<LPE>(P, T, cur, i, ch, A, smem);
+    int r;
+    if constexpr (LPE == 0) r = gen_child_small(P, T, cur, i, ch, A, smem);
+    else r = gen_child<LPE>(P, T, cur, i, ch, A, smem);
     if (r == 2 && split_mode && cur == top) {
       // Alg 4 L25: hand the child to the task queue as a self-contained subtask
       PH_START(A);
@@ -762,11 +924,13 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
   }
 }
 
-__device__ void dispatch_task(const Params& P, const TaskCtx& T, uint32_t* top, uint32_t* lo, uint32_t* hi,
+__device__ void dispatch_task(const Params& P, TaskCtx& T, uint32_t* top, uint32_t* lo, uint32_t* hi,
                               uint32_t lmap, Acc& A, unsigned long long* smem) {
-  if (T.W <= 1) run_task<1>(P, T, top, lo, hi, lmap, A, smem);
-  else if (T.W <= 2) run_task<2>(P, T, top, lo, hi, lmap, A, smem);
-  else if (T.W <= 4) run_task<4>(P, T, top, lo, hi, lmap, A, smem);
+  if (T.W <= 2) {
+    small_task_init(P, T, lmap);
+    run_task<0>(P, T, top, lo, hi, lmap, A, smem);
+  }
+  else if (T.W <= 4) run_task<4>(P, T, top, lo, hi, lmap, A, smem);  // W > 2 from here
   else if (T.W <= 8) run_task<8>(P, T, top, lo, hi, lmap, A, smem);
   else if (T.W <= 16) run_task<16>(P, T, top, lo, hi, lmap, A, smem);
   else run_task<32>(P, T, top, lo, hi, lmap, A, smem);
@@ -961,8 +1125,8 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
         __threadfence();  // rows / columns were built with atomics: drop stale L1 lines
       }
       PH_STOP(A, 11);
-      for (uint32_t w = lane; w < W; w += 32) {
-        const uint32_t bits = l - w * 32;
+      for (uint32_t w = lane; w < W4; w += 32) {
+        const uint32_t bits = w < W ? l - w * 32 : 0u;
         rec[kHdr + w] = bits >= 32 ? GMBE_FULL : ((1u << bits) - 1u);
       }
       if (lane == 0) {
