@@ -171,6 +171,7 @@ def main():
     import torch
     import torch.distributed as dist
     import paper_conf_sc_panhlzwc23_b200 as gmbe
+    from paper_conf_sc_panhlzwc23_b200 import dist as gdist
     from gmbe_inputs import make_config, graph_stats
 
     ws, rank, local = _dist()
@@ -193,11 +194,8 @@ def main():
         r = g.enumerate(part=part, stream=stream)
         g.free()
         kernel_ms.append(r.kernel_ms)
-        res = torch.tensor([r.count, r.checksum - (1 << 64) if r.checksum >= 1 << 63 else r.checksum,
-                            r.nodes, r.nonmax], dtype=torch.int64, device=dev)
-        if ws > 1:
-            dist.all_reduce(res)  # the only cross-GPU exchange (NVLink / NVSwitch)
-        return res
+        # the only cross-GPU exchange: one NCCL all-reduce of the int64-viewed totals (N > 1)
+        return gdist.allreduce_result(r, device=dev)
 
     # canonical work of this shard (identical in every schedule; reported by every run)
     g = gmbe.load(nu, nv, e_dev, device=local, stream=stream)
@@ -237,10 +235,7 @@ def main():
         g = gmbe.load(nu, nv, e_host.numpy(), device=local, stream=stream)
         r = g.enumerate(part=part, stream=stream)
         g.free()
-        rr = torch.tensor([r.count], dtype=torch.int64, device=dev)
-        if ws > 1:
-            dist.all_reduce(rr)
-        total_e2e = int(rr.item())
+        total_e2e = gdist.allreduce_result(r, device=dev)["count"]
         e1.record(stream)
         e1.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
@@ -252,8 +247,8 @@ def main():
     if ws > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     t_step, t_e2e = float(tt[0]), float(tt[1])
-    count = int(res[0].item())
-    checksum = int(res[1].item()) % (1 << 64)
+    count = res["count"]
+    checksum = res["checksum"]
     assert total_e2e == count
 
     if rank == 0:
