@@ -15,7 +15,7 @@ from dataclasses import dataclass, field
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgmbe.so")
+LIB_PATH = os.environ.get("GMBE_LIB") or os.path.join(_HERE, "libgmbe.so")  # GMBE_LIB: experiments only
 if not os.path.exists(LIB_PATH):
     raise ImportError("libgmbe.so is not built (run `python -c 'import __graft_entry__ as e; e.build()'`); "
                       "there is no CPU fallback")

@@ -1178,7 +1178,10 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
   __syncwarp();
 }
 
-__global__ void __launch_bounds__(256) k_enum(const Params P) {
+#ifndef GMBE_MIN_BLOCKS
+#define GMBE_MIN_BLOCKS 3  // 80 registers: 24 resident warps per SM (measured best on gh_work)
+#endif
+__global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
   __shared__ unsigned long long s_sort[8][kSmemSort];
   const uint32_t lane = lane_id();
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
