@@ -189,10 +189,17 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)          # > 126 MB L2
     part = (rank, ws)
 
+    host_ms = {"load": [], "enumerate": []}
+
     def step(edges, kernel_ms):
+        t0 = time.perf_counter()
         g = gmbe.load(nu, nv, edges, device=local, stream=stream)
+        t1 = time.perf_counter()
         r = g.enumerate(part=part, stream=stream)
+        t2 = time.perf_counter()
         g.free()
+        host_ms["load"].append(1e3 * (t1 - t0))
+        host_ms["enumerate"].append(1e3 * (t2 - t1))
         kernel_ms.append(r.kernel_ms)
         # the only cross-GPU exchange: one NCCL all-reduce of the int64-viewed totals (N > 1)
         return gdist.allreduce_result(r, device=dev)
@@ -279,6 +286,7 @@ def main():
                        "l2": "flushed between steps (256 MiB memset)",
                        "step": "device CSR build + enumerate (+ all-reduce)"},
             "kernel_ms": k_rank,
+            "host_wall_ms": {k: round(sum(v[-a.steps:]) / max(1, len(v[-a.steps:])), 3) for k, v in host_ms.items()},
             "e2e": {"value": count / (t_e2e * 1e-3), "unit": "bicliques/s",
                     "h2d_bytes_per_step": int(m * 8), "d2h_bytes_per_step": CTRL_D2H_BYTES},
             "gpu_launches": int(launches),

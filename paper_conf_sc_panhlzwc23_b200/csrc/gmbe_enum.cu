@@ -1284,6 +1284,9 @@ struct Workspace {
   size_t arena_bytes = 0;
   uint64_t layout[4] = {0, 0, 0, 0};  // tmax, omax, arena_words, nwarps of the clean tables
   bool clean = false;
+  uint64_t tmax = 0, omax = 0, dyn = 0, nwarps = 0, pool_auto = 0;  // cached sizing
+  bool dyn_capped = false;
+  int sms = 0, bps_max = 0;
   void* pool = nullptr;
   size_t pool_bytes = 0;
   void* rings = nullptr;
@@ -1376,43 +1379,65 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   } ret{Wp};
   Workspace& W = *Wp;
 
-  int sms = 0;
-  GMBE_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, G->device));
+  if (W.sms == 0) {  // per-device constants, queried once per workspace
+    GMBE_CUDA_TRY(cudaDeviceGetAttribute(&W.sms, cudaDevAttrMultiProcessorCount, G->device));
+    GMBE_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&W.bps_max, k_enum, 256, 0));
+  }
   uint32_t wps = o.warps_per_sm ? o.warps_per_sm : 32;
   if (wps < 8) wps = 8;
   if (wps > 64) wps = 64;
-  int bps_max = 0;
-  GMBE_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps_max, k_enum, 256, 0));
   uint32_t bps = wps / 8;
-  if ((int)bps > bps_max) bps = bps_max;
+  if ((int)bps > W.bps_max) bps = W.bps_max;
   if (bps < 1) bps = 1;
-  const uint32_t blocks = (uint32_t)sms * bps;
+  const uint32_t blocks = (uint32_t)W.sms * bps;
   const uint64_t nwarps = (uint64_t)blocks * 8;
 
   // per-warp arena: clean hash table sized for the largest root's wedges, its occupied list, and
-  // the dynamic region (root record, node stack), bounded by free memory
+  // the dynamic region (root record, node stack, Γ index), bounded by free memory.  A cached layout
+  // that already satisfies this graph is reused as is (its tables are clean; no re-initialisation).
   const uint64_t wb = (uint64_t)g.wedge_bound + 64;
   uint64_t tmax = 64;
   while (tmax < 2 * wb) tmax <<= 1;
-  const uint64_t omax = (wb + 3) & ~3ull;
-  const uint64_t fixed = 3 * tmax + omax + 8;
-  uint64_t dyn = o.arena_words;
-  if (!dyn) {
-    // root record + node stack + Γ columns (|L_r| x |X|/32, capped at 2M words)
-    const uint64_t cols_bound = std::min<uint64_t>((uint64_t)g.delta_v * (wb / 32 + 1), 1u << 21);
-    const uint64_t want = (uint64_t)g.rec_bound * 4 + 4 * wb + 2 * cols_bound + (1u << 18);
-    size_t fr = 0, tot = 0;
-    GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
-    const uint64_t cap_total = (uint64_t)(fr * 0.5) / 4 / nwarps;
-    const uint64_t cap = cap_total > fixed + (1u << 16) ? cap_total - fixed : (1u << 16);
-    dyn = want < cap ? want : cap;
+  uint64_t omax = (wb + 3) & ~3ull;
+  const uint64_t cols_bound = std::min<uint64_t>((uint64_t)g.delta_v * (wb / 32 + 1), 1u << 21);
+  const uint64_t dyn_want = o.arena_words ? o.arena_words
+                                          : (uint64_t)g.rec_bound * 4 + 4 * wb + 2 * cols_bound + (1u << 18);
+  uint64_t arena_words;
+  if (W.arena && W.nwarps == nwarps && W.tmax >= tmax && W.omax >= omax &&
+      (W.dyn >= dyn_want || (!o.arena_words && W.dyn_capped))) {
+    tmax = W.tmax;
+    omax = W.omax;
+    arena_words = W.layout[2];
+  } else {
+    const uint64_t fixed = 3 * tmax + omax + 8;
+    uint64_t dyn = dyn_want;
+    bool capped = false;
+    if (!o.arena_words) {
+      size_t fr = 0, tot = 0;
+      GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
+      fr += W.arena_bytes;  // this workspace's arena is about to be replaced
+      const uint64_t cap_total = (uint64_t)(fr * 0.5) / 4 / nwarps;
+      const uint64_t cap = cap_total > fixed + (1u << 16) ? cap_total - fixed : (1u << 16);
+      if (dyn > cap) {
+        dyn = cap;
+        capped = true;
+      }
+    }
+    arena_words = (fixed + dyn + 3) & ~3ull;
+    W.tmax = tmax;
+    W.omax = omax;
+    W.dyn = dyn;
+    W.dyn_capped = capped;
+    W.nwarps = nwarps;
   }
-  const uint64_t arena_words = (fixed + dyn + 3) & ~3ull;
   uint64_t pool_words = o.pool_words;
-  if (!pool_words) {  // task pool: subtasks + shared columns, never reused within a call
-    size_t fr = 0, tot = 0;
-    GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
-    pool_words = std::min<uint64_t>(1ull << 30, (uint64_t)(fr * 0.2) / 4);
+  if (!pool_words) {  // task pool: subtasks + shared Γ indexes, never reused within a call
+    if (!W.pool_auto) {
+      size_t fr = 0, tot = 0;
+      GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
+      W.pool_auto = std::min<uint64_t>(1ull << 30, (uint64_t)(fr * 0.2) / 4);
+    }
+    pool_words = W.pool_auto;
   }
   pool_words = (pool_words + 3) & ~3ull;
   uint32_t cap = 1;

@@ -1,0 +1,53 @@
+"""Summarise an ncu --set full report of k_enum: key metrics, stall mix, top source lines.
+    python scripts/ncu_summary.py gpurun_out/prof.ncu-rep [--json out.json] [--src N]"""
+import csv
+import io
+import json
+import subprocess
+import sys
+
+rep = sys.argv[1]
+out_json = sys.argv[sys.argv.index("--json") + 1] if "--json" in sys.argv else None
+nsrc = int(sys.argv[sys.argv.index("--src") + 1]) if "--src" in sys.argv else 25
+
+
+def ncu(*a):
+    return subprocess.run(["ncu", "-i", rep] + list(a), capture_output=True, text=True).stdout
+
+
+rows = list(csv.reader(io.StringIO(ncu("--page", "raw", "--csv"))))
+hdr, units, vals = rows[0], rows[1], rows[2]
+m = {h: (v, u) for h, v, u in zip(hdr, vals, units)}
+keys = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum", "lts__t_bytes.sum",
+        "sm__cycles_active.avg", "sm__cycles_active.max", "sm__cycles_active.min",
+        "smsp__thread_inst_executed_per_inst_executed.ratio", "sm__warps_active.avg.pct_of_peak_sustained_active",
+        "smsp__issue_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
+        "launch__grid_size", "launch__block_size", "l1tex__t_sector_hit_rate.pct", "lts__t_sector_hit_rate.pct",
+        "dram__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum"]
+summ = {k: m[k][0] + " " + m[k][1] for k in keys if k in m}
+st = {h[len("smsp__pcsamp_warps_issue_stalled_"):]: float(v.replace(",", "") or 0) for h, (v, u) in m.items()
+      if h.startswith("smsp__pcsamp_warps_issue_stalled_") and not h.endswith("not_issued")}
+tot = sum(st.values()) or 1
+summ["stall_mix_pct"] = {k: round(100 * v / tot, 1) for k, v in sorted(st.items(), key=lambda x: -x[1]) if v / tot > 0.005}
+for k, v in summ.items():
+    print(k, v)
+src = list(csv.reader(io.StringIO(ncu("--page", "source", "--csv", "--print-source", "cuda,sass"))))
+h = src[2]
+iS = h.index("Warp Stall Sampling (All Samples)")
+agg, total = {}, 0
+for r in src[3:]:
+    if len(r) > iS and r[0] not in ("-", "") and r[2] == "-":
+        try:
+            n = int(r[iS].replace(",", ""))
+        except ValueError:
+            continue
+        agg[(int(r[0]), r[1].strip())] = n
+        total += n
+top = sorted(agg.items(), key=lambda x: -x[1])[:nsrc]
+print("top source lines by stall samples:")
+for (ln, code), n in top:
+    print("%5d %5.1f%%  %s" % (ln, 100.0 * n / total, code[:100]))
+summ["top_lines"] = [[ln, round(100.0 * n / total, 2), code[:100]] for (ln, code), n in top]
+if out_json:
+    with open(out_json, "w") as f:
+        json.dump(summ, f, indent=1)
