@@ -1477,7 +1477,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.hu_side = g.swapped ? 1 : 0;
   P.arena = (uint32_t*)W.arena;
   P.arena_words = arena_words;
-  P.col_budget = dyn / 2;
+  P.col_budget = W.dyn / 2;
   P.tmax = (uint32_t)tmax;
   P.omax = (uint32_t)omax;
   P.rbuf = want_out ? (uint32_t*)W.rbuf : nullptr;
