@@ -7,6 +7,7 @@ SRC = [os.path.join(HERE, "csrc", f) for f in ("gmbe_api.cu", "gmbe_graph.cu", "
 DEPS = SRC + [os.path.join(HERE, "csrc", "gmbe_internal.cuh"),
               os.path.join(os.path.dirname(HERE), "include", "gmbe.h")]
 LIB = os.path.join(HERE, "libgmbe.so")
+LIB_PROF = os.path.join(HERE, "libgmbe_prof.so")  # phase-profiling variant (-DGMBE_PROFILE)
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
               "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-v"]
 
@@ -18,20 +19,25 @@ def nvcc():
     return "nvcc"
 
 
-def build(force=False, verbose=False):
-    """Compile every CUDA source into libgmbe.so (skipped when up to date)."""
-    if not force and os.path.exists(LIB):
-        t = os.path.getmtime(LIB)
+def build(force=False, verbose=False, profile=False):
+    """Compile every CUDA source into libgmbe.so (and, with profile=True, libgmbe_prof.so).
+    Skipped when up to date."""
+    if profile:
+        build(force, verbose)
+    lib = LIB_PROF if profile else LIB
+    if not force and os.path.exists(lib):
+        t = os.path.getmtime(lib)
         if all(os.path.getmtime(d) <= t for d in DEPS):
-            return LIB
-    tmp = LIB + ".tmp.%d" % os.getpid()
-    cmd = [nvcc()] + NVCC_FLAGS + ["-o", tmp] + SRC
+            return lib
+    tmp = lib + ".tmp.%d" % os.getpid()
+    cmd = [nvcc()] + NVCC_FLAGS + (["-DGMBE_PROFILE"] if profile else []) + ["-o", tmp] + SRC
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError("nvcc failed:\n" + r.stdout + r.stderr)
-    with open(os.path.join(HERE, "ptxas_report.txt"), "w") as f:
-        f.write(r.stdout + r.stderr)
+    if not profile:
+        with open(os.path.join(HERE, "ptxas_report.txt"), "w") as f:
+            f.write(r.stdout + r.stderr)
     if verbose:
         print(r.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib

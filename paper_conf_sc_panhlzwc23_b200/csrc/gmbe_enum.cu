@@ -82,11 +82,15 @@ struct Params {
 
 struct Acc {
   unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
-  unsigned long long ph[16];  // profiling: SM cycles per phase (opts.phase_cycles)
+#ifdef GMBE_PROFILE
+  unsigned long long ph[16];  // profiling build only: SM cycles per phase (opts.phase_cycles)
   long long t0;
+#endif
 };
-// phase profiling (no-op unless P.profile): 0 root wedge pass, 1 classify, 2 sort, 3 root record +
-// columns, 4 candidate scan, 5 maximality, 6 emit, 7 task queue
+// Phase profiling (libgmbe_prof.so, built with -DGMBE_PROFILE; compiled out of libgmbe.so):
+// 0 root wedge pass, 1 classify, 2 sort, 3 root finish, 4 candidate scan, 5 maximality, 6 emit,
+// 7 task queue, 8.. root sub-phases (names in the Python binding's PHASES)
+#ifdef GMBE_PROFILE
 #define PH_START(A) \
   if (P.profile) (A).t0 = clock64()
 #define PH_STOP(A, k)                                   \
@@ -95,6 +99,14 @@ struct Acc {
     (A).ph[k] += (unsigned long long)(_t - (A).t0);     \
     (A).t0 = _t;                                        \
   }
+#else
+#define PH_START(A) \
+  do {              \
+  } while (0)
+#define PH_STOP(A, k) \
+  do {                \
+  } while (0)
+#endif
 
 // per-task constants (warp-uniform)
 struct TaskCtx {
@@ -115,6 +127,7 @@ struct TaskCtx {
   // small_task_init: Γ-list offsets / lengths and the checksum hashes of the universe vertices
   uint32_t go0, go1, gl0, gl1;
   unsigned long long hu0, hu1;
+  const uint32_t* gxl;  // gx: base of the per-vertex 2-hop lists
 };
 
 // per-warp memory
@@ -128,7 +141,11 @@ struct WarpMem {
   unsigned long long* sm_sort;  // this warp's shared-memory sort slice
 };
 
-__device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ uint32_t lane_id() {
+  uint32_t l;
+  asm("mov.u32 %0, %%laneid;" : "=r"(l));  // non-volatile: the compiler may CSE it
+  return l;
+}
 __device__ __forceinline__ uint32_t lanemask_lt() { return (1u << lane_id()) - 1u; }
 __device__ __forceinline__ uint32_t r4(uint32_t x) { return (x + 3u) & ~3u; }
 __device__ __forceinline__ uint32_t* align4(uint32_t* p) {
@@ -726,9 +743,11 @@ __device__ void small_task_init(const Params& P, TaskCtx& T, uint32_t lmap) {
   T.go0 = T.go1 = T.gl0 = T.gl1 = 0;
   T.hu0 = lane < lmap ? gmbe_hid(T.map[lane], P.hu_side) : 0ull;
   T.hu1 = lane + 32 < lmap ? gmbe_hid(T.map[lane + 32], P.hu_side) : 0ull;
+  T.gxl = nullptr;
   if (T.gx) {
     const uint32_t* coff = T.gx + 4 + 2 * T.gx[0];
     const uint32_t l = T.gx[1];
+    T.gxl = coff + r4(l + 1);
     if (lane < l) {
       T.go0 = coff[lane];
       T.gl0 = coff[lane + 1] - T.go0;
@@ -750,9 +769,8 @@ __device__ __forceinline__ bool gamma_gx_small(const TaskCtx& T, unsigned long l
   const uint32_t js = key & 127u, len = key >> 7;
   if (len + 1 == rlen) return true;  // |Γ(L')| <= deg(u*) = len + 1
   const uint32_t off = __shfl_sync(GMBE_FULL, js < 32 ? T.go0 : T.go1, js & 31);
-  const uint32_t nx = T.gx[0];
   const unsigned long long* xrow = (const unsigned long long*)(T.gx + 4);
-  const uint32_t* lst = T.gx + 4 + 2 * nx + r4(T.gx[1] + 1) + off;
+  const uint32_t* lst = T.gxl + off;
   uint32_t count = 1;  // v_s
   for (uint32_t b = 0; b < len; b += 32) {
     bool full = false;
@@ -1272,8 +1290,10 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
     atomicAdd(&c->abytes, A.abytes);
     atomicAdd(&c->splits, A.splits);
     atomicAdd(&c->tasks, A.tasks);
+#ifdef GMBE_PROFILE
     if (P.profile)
       for (int k = 0; k < 16; k++) atomicAdd(&c->phase[k], A.ph[k]);
+#endif
   }
 }
 

@@ -6,7 +6,11 @@ import os
 import numpy as np
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-import torch  # noqa: E402
+# the phase-profiling build (libgmbe_prof.so, -DGMBE_PROFILE); build it with
+#   python -c "import importlib.util as u; ..._build.build(profile=True)"  (see __graft_entry__)
+os.environ.setdefault("GMBE_LIB", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                                               "paper_conf_sc_panhlzwc23_b200", "libgmbe_prof.so"))
+import torch  # noqa: E402,F401
 import paper_conf_sc_panhlzwc23_b200 as gmbe  # noqa: E402
 from gmbe_inputs import make_config  # noqa: E402
 
