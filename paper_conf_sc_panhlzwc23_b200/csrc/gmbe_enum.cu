@@ -307,7 +307,7 @@ __device__ void warp_sort_keys(unsigned long long* a, uint32_t n, unsigned long 
     __syncwarp();
     return;
   }
-  if (next_pow2(n) <= kSmemSort) {
+  if (smem && next_pow2(n) <= kSmemSort) {
     for (uint32_t j = lane; j < n; j += 32) smem[j] = a[j];
     __syncwarp();
     warp_bitonic64(smem, n);
@@ -896,6 +896,149 @@ __device__ __forceinline__ bool heavy(const Params& P, uint32_t l, uint32_t nC) 
 
 // Walk the subtree of `top` (Alg 2) on the node stack [stack_lo, stack_hi) -- or, when the task is
 // heavy (Alg 4 L17), hand top's children to the task queue as self-contained subtasks.
+// ---------------------------------------------------------------- register-resident subtrees
+// A node with <= 32 candidates over a <= 64-bit universe: every descendant's candidates are a subset
+// of its candidates, so lane j keeps candidate j's row / id / hV for the whole subtree and a node is
+// just (L mask, candidate lane mask).  Alg 2 on that representation: child via lane i -> L' = L & row_i;
+// later = candidate lanes > i; k' = popc(row & L'), k = popc(row & L); Thm 4.1 clears the lanes with
+// k' == k from the node; R' absorbs k' == |L'|; C' = 0 < k' < |L'|.  Levels (<= 32) live in the warp's
+// shared-memory slice.  `split_top`: the node is a heavy task top -- publish its children (Alg 4 L25).
+struct RegLevel {
+  unsigned long long L, SR;
+  uint32_t C, next, rlen, pad;
+};
+__device__ __forceinline__ unsigned long long shfl64(unsigned long long x, uint32_t src) {
+  const uint32_t lo = __shfl_sync(GMBE_FULL, (uint32_t)x, src);
+  const uint32_t hi = __shfl_sync(GMBE_FULL, (uint32_t)(x >> 32), src);
+  return ((unsigned long long)hi << 32) | lo;
+}
+__device__ void run_reg(const Params& P, const TaskCtx& T, const uint32_t* rec, uint32_t lmap, Acc& A,
+                        RegLevel* st, uint32_t* scratch, const uint32_t* scratch_end, bool split_top,
+                        unsigned long long* smem) {
+  const uint32_t lane = lane_id();
+  const bool w2 = T.W == 2;
+  const uint32_t nC = rec[0];
+  unsigned long long row = 0, hvj = 0;
+  uint32_t id = 0;
+  if (lane < nC) {
+    const uint4 x = ((const uint4*)(rec + kHdr + 4))[lane];
+    row = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
+    id = w2 ? x.z : x.y;
+    hvj = P.g.hv[id];
+  }
+  unsigned long long L = ((unsigned long long)rec[kHdr + 1] << 32) | rec[kHdr];
+  unsigned long long SR = ((unsigned long long)rec[7] << 32) | rec[6];
+  uint32_t C = nC >= 32 ? GMBE_FULL : ((1u << nC) - 1u), next = 0, rlen = rec[5];
+  int d = 0;
+  while (true) {
+    const uint32_t avail = next >= 32 ? 0u : (C & ~((1u << next) - 1u));
+    if (!avail) {  // pop (Alg 2 L4)
+      if (d == 0) break;
+      d--;
+      L = st[d].L;
+      SR = st[d].SR;
+      C = st[d].C;
+      next = st[d].next;
+      rlen = st[d].rlen;
+      continue;
+    }
+    const uint32_t i = __ffs(avail) - 1;
+    next = i + 1;
+    const unsigned long long lp = L & shfl64(row, i);  // L' = L_p ∩ N(v')
+    const uint32_t lc = __popcll(lp);
+    const uint32_t later = i >= 31 ? 0u : (C & ~((2u << i) - 1u));
+    const bool inl = (later >> lane) & 1u;
+    const uint32_t kp = __popcll(row & L), kc = __popcll(row & lp);
+    const uint32_t pr = __ballot_sync(GMBE_FULL, inl && P.prune && kc == kp);
+    const uint32_t ab = __ballot_sync(GMBE_FULL, inl && kc == lc);
+    const uint32_t cd = __ballot_sync(GMBE_FULL, inl && kc > 0 && kc < lc);
+    C &= ~pr;  // Thm 4.1
+    A.nodes++;
+    A.abytes += 4ull * (lc + __reduce_add_sync(GMBE_FULL, inl ? kp : 0u));
+    const uint32_t rl = rlen + 1 + __popc(ab);
+    bool maximal;
+    if (lc == 1) {
+      const uint32_t u = T.map[__ffsll(lp) - 1];
+      maximal = P.g.off_u[u + 1] - P.g.off_u[u] == rl;
+    } else if (T.gx) {
+      maximal = gamma_gx_small(T, lp, rl);
+    } else {
+      if (lane == 0) {
+        scratch[0] = (uint32_t)lp;
+        scratch[1] = (uint32_t)(lp >> 32);
+      }
+      __syncwarp();
+      maximal = gamma_is_r(P, scratch, T.W, T.map, lc, rl, (unsigned long long*)(scratch + 4), nullptr);
+    }
+    if (!maximal) {
+      A.nonmax++;
+      continue;
+    }
+    // Output(L', R') (Alg 2 L15)
+    const uint32_t idi = __shfl_sync(GMBE_FULL, id, i);
+    const unsigned long long srn = SR + shfl64(hvj, i) + warp_sum64r(((ab >> lane) & 1u) ? hvj : 0ull);
+    const unsigned long long sl =
+        warp_sum64r(((lp >> lane) & 1ull ? T.hu0 : 0ull) + ((lp >> (lane + 32)) & 1ull ? T.hu1 : 0ull));
+    A.count++;
+    A.checksum += pair_hash(P, sl, srn);
+    if (P.per_root && lane == 0) atomicAdd(P.per_root + T.root, 1ull);
+    if (T.rlist) {
+      if (lane == 0) T.rlist[rlen] = idi;
+      if ((ab >> lane) & 1u) T.rlist[rlen + 1 + __popc(ab & lanemask_lt())] = id;
+      if (lane == 0) {
+        scratch[0] = (uint32_t)lp;
+        scratch[1] = (uint32_t)(lp >> 32);
+      }
+      __syncwarp();
+      if (P.out_ids) write_record(P, scratch, T.W, T.map, nullptr, lc, T.rlist, rl);
+    }
+    if (!cd) continue;
+    if (split_top && d == 0) {
+      // publish the child as a subtask: node record [hdr | L' | entries (row & L', id, k')]
+      const uint32_t words = kHdr + 4 + 4 * __popc(cd);
+      if (scratch + words <= scratch_end) {
+        uint4* ce = (uint4*)(scratch + kHdr + 4);
+        if ((cd >> lane) & 1u) {
+          const unsigned long long xr = row & lp;
+          ce[__popc(cd & lanemask_lt())] = w2 ? make_uint4((uint32_t)xr, (uint32_t)(xr >> 32), id, kc)
+                                              : make_uint4((uint32_t)xr, id, kc, 0);
+        }
+        if (lane == 0) {
+          scratch[0] = __popc(cd);
+          scratch[1] = 0;
+          scratch[2] = lc;
+          scratch[3] = 0;
+          scratch[4] = kNone;
+          scratch[5] = rl;
+          scratch[6] = (uint32_t)srn;
+          scratch[7] = (uint32_t)(srn >> 32);
+          scratch[kHdr] = (uint32_t)lp;
+          scratch[kHdr + 1] = (uint32_t)(lp >> 32);
+          scratch[kHdr + 2] = 0;
+          scratch[kHdr + 3] = 0;
+        }
+        __syncwarp();
+        if (task_publish(P, T, lmap, T.rlist ? rl : 0, scratch, words, A)) continue;
+      }
+    }
+    // push (Alg 2 L16)
+    if (lane == 0) {
+      st[d].L = L;
+      st[d].SR = SR;
+      st[d].C = C;
+      st[d].next = next;
+      st[d].rlen = rlen;
+    }
+    __syncwarp();
+    d++;
+    L = lp;
+    SR = srn;
+    C = cd;
+    next = 0;
+    rlen = rl;
+  }
+}
+
 template <int LPE>
 __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint32_t* stack_lo, uint32_t* stack_hi,
                          uint32_t lmap, Acc& A, unsigned long long* smem) {
@@ -904,6 +1047,12 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
   uint32_t* sp = stack_lo;  // first free word
   const bool split_mode = heavy(P, top[2], top[0]);
   if (split_mode) A.splits++;
+  if constexpr (LPE == 0) {
+    if (top[0] <= 32) {  // the whole task fits the register-resident DFS
+      run_reg(P, T, top, lmap, A, (RegLevel*)smem, stack_lo, stack_hi, split_mode, smem);
+      return;
+    }
+  }
   while (true) {
     __syncwarp();
     const uint32_t i = cur[3];
@@ -929,6 +1078,12 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
       const bool done = task_publish(P, T, lmap, T.rlist ? ch[5] : 0, ch, rec_words(T, ch), A);
       PH_STOP(A, 7);
       if (done) continue;
+    }
+    if constexpr (LPE == 0) {
+      if (r == 2 && ch[0] <= 32) {  // the child's subtree fits the register-resident DFS
+        run_reg(P, T, ch, lmap, A, (RegLevel*)smem, align4(ch + rec_words(T, ch)), stack_hi, false, smem);
+        continue;
+      }
     }
     if (r == 2) {  // push (Alg 2 L16)
       if (lane == 0) {
