@@ -783,8 +783,11 @@ __device__ __forceinline__ bool gamma_gx_small(const TaskCtx& T, unsigned long l
 
 // gen_child for W <= 2: one lane per candidate entry, loaded as one 16-byte vector
 // ({row, id, k, -} for W = 1, {row_lo, row_hi, id, k} for W = 2); L' and rows as 64-bit masks.
+// dom != null: `par` is a published split node (read-only, shared by several warps) and the later
+// candidates of child i are {k > i : dom[k] >= i} -- the Thm 4.1 marks of the earlier siblings,
+// precomputed by split_parallel -- so no compaction / marking happens here.
 __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par, uint32_t i, uint32_t* ch, Acc& A,
-                               unsigned long long* smem) {
+                               unsigned long long* smem, const uint32_t* dom = nullptr) {
   const uint32_t lane = lane_id();
   const bool w2 = T.W == 2;
   const uint32_t nC = par[0];
@@ -808,7 +811,7 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
   const uint32_t rl_base = par[5] + 1;
   for (uint32_t base = i + 1; base < nC; base += 32) {
     const uint32_t j = base + lane;
-    const bool in = j < nC;
+    const bool in = j < nC && (!dom || dom[j] >= i);
     uint4 x = make_uint4(0, 0, 0, 0);
     if (in) x = pent[j];
     const unsigned long long row = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
@@ -829,14 +832,16 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
       cent[nCc + __popc(bc & lanemask_lt())] =
           w2 ? make_uint4((uint32_t)xr, (uint32_t)(xr >> 32), id, cnt) : make_uint4((uint32_t)xr, id, cnt, 0);
     nCc += __popc(bc);
-    const uint32_t bs = __ballot_sync(GMBE_FULL, surv);
-    const uint32_t spos = i + 1 + nsurv + __popc(bs & lanemask_lt());
-    nsurv += __popc(bs);
-    __syncwarp();
-    if (surv && spos != j) pent[spos] = x;
-    __syncwarp();
+    if (!dom) {
+      const uint32_t bs = __ballot_sync(GMBE_FULL, surv);
+      const uint32_t spos = i + 1 + nsurv + __popc(bs & lanemask_lt());
+      nsurv += __popc(bs);
+      __syncwarp();
+      if (surv && spos != j) pent[spos] = x;
+      __syncwarp();
+    }
   }
-  if (lane == 0) par[0] = i + 1 + nsurv;
+  if (lane == 0 && !dom) par[0] = i + 1 + nsurv;
   A.nodes++;
   A.abytes += 4ull * (lc + warp_sum64r(later_k));
   const uint32_t rlen = par[5] + 1 + r_abs;
@@ -1039,6 +1044,96 @@ __device__ void run_reg(const Params& P, const TaskCtx& T, const uint32_t* rec, 
   }
 }
 
+// ---------------------------------------------------------------- parallel split (a7)
+// Thm 4.1 at a node prunes candidate c for the later siblings of child i iff k'(c) = k(c), i.e.
+// row(c) ⊆ row(c_i).  Subset domination is transitive, so c_k is pruned before its own turn iff some
+// earlier candidate's row contains row(c_k), and the earliest such one, dom(k), is itself generated.
+// Hence: children = G = {j : dom(j) undefined}, and the later set of child j is {k > j : dom(k) >= j}.
+// split_parallel computes dom / G for a heavy task top (universe <= 64 bits), publishes the node once
+// (read-only) and enqueues range descriptors over G, so sibling children are generated by different
+// warps instead of one sequential loop (the tree, and every counter, is unchanged).
+constexpr uint32_t kDescMagic = 0xFFFFFFF0u;
+constexpr uint32_t kDescChildren = 4;  // children per descriptor
+__device__ bool split_parallel(const Params& P, const TaskCtx& T, const uint32_t* top, uint32_t lmap, Acc& A,
+                               uint32_t* scratch, const uint32_t* scratch_end) {
+  const uint32_t lane = lane_id();
+  const bool w2 = T.W == 2;
+  const uint32_t n = top[0];
+  const uint32_t words = kHdr + 4 + 4 * n;  // node record (W <= 2: 16-byte entries)
+  uint32_t* dom = scratch;
+  uint32_t* G = dom + r4(n);
+  if (G + r4(n) + 64 > scratch_end || !queue_room(P)) return false;
+  const uint4* ent = (const uint4*)(top + kHdr + 4);
+  uint32_t ng = 0;
+  for (uint32_t kb = 0; kb < n; kb += 32) {
+    const uint32_t k = kb + lane;
+    unsigned long long rk = 0;
+    if (k < n) {
+      const uint4 x = ent[k];
+      rk = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
+    }
+    uint32_t d = k < n ? kNone : 0u;
+    // dominators among the generated candidates of earlier chunks
+    for (uint32_t t = 0; t < ng && __any_sync(GMBE_FULL, d == kNone); t++) {
+      const uint32_t gi = G[t];
+      const uint4 x = ent[gi];
+      const unsigned long long ri = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
+      if (d == kNone && (ri & rk) == rk) d = gi;
+    }
+    // within the chunk, in order
+    for (uint32_t t = 0; t < 32 && kb + t < n; t++) {
+      const bool gen_t = __shfl_sync(GMBE_FULL, d, t) == kNone;
+      if (gen_t) {
+        const unsigned long long rt = shfl64(rk, t);
+        if (lane > t && d == kNone && (rt & rk) == rk) d = kb + t;
+      }
+    }
+    if (k < n) dom[k] = d;
+    const uint32_t bg = __ballot_sync(GMBE_FULL, k < n && d == kNone);
+    if (k < n && d == kNone) G[ng + __popc(bg & lanemask_lt())] = k;
+    ng += __popc(bg);
+    __syncwarp();
+  }
+  // publish: task record (map | R list | node | dom | G) + descriptors over G
+  const uint32_t rlen = T.rlist ? top[5] : 0;
+  const uint32_t node_off = task_node_off(lmap, rlen);
+  const uint32_t total = node_off + words + r4(n) + r4(ng);
+  const uint32_t nd = (ng + kDescChildren - 1) / kDescChildren;
+  const uint32_t off16 = pool_alloc(P, r4(total) + 4 * nd);
+  if (off16 == kNone) return false;
+  uint32_t* s = pool_ptr(P, off16);
+  for (uint32_t j = lane; j < lmap; j += 32) s[kHdr + j] = T.map[j];
+  if (T.rlist)
+    for (uint32_t j = lane; j < rlen; j += 32) s[kHdr + r4(lmap) + j] = T.rlist[j];
+  for (uint32_t j = lane; j < words; j += 32) s[node_off + j] = top[j];
+  uint32_t* sd = s + node_off + words;
+  for (uint32_t j = lane; j < n; j += 32) sd[j] = dom[j];
+  for (uint32_t j = lane; j < ng; j += 32) sd[r4(n) + j] = G[j];
+  uint32_t* desc = s + r4(total);
+  for (uint32_t t = lane; t < nd; t += 32) {
+    desc[4 * t] = kDescMagic;
+    desc[4 * t + 1] = off16;
+    desc[4 * t + 2] = t * kDescChildren;
+    desc[4 * t + 3] = min(ng, (t + 1) * kDescChildren);
+  }
+  if (lane == 0) {
+    s[0] = T.W;
+    s[1] = lmap;
+    s[2] = T.root;
+    s[3] = rlen;
+    s[4] = node_off;
+    s[5] = T.auxref;
+    s[6] = T.ncw;
+    s[7] = T.auxref ? (T.gx ? 2u : 1u) : 0u;
+  }
+  A.tasks += nd;
+  __threadfence();
+  __syncwarp();
+  const uint32_t desc16 = off16 + r4(total) / 4;
+  for (uint32_t t = lane; t < nd; t += 32) queue_push(P, desc16 + t);
+  return true;
+}
+
 template <int LPE>
 __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint32_t* stack_lo, uint32_t* stack_hi,
                          uint32_t lmap, Acc& A, unsigned long long* smem) {
@@ -1048,6 +1143,7 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
   const bool split_mode = heavy(P, top[2], top[0]);
   if (split_mode) A.splits++;
   if constexpr (LPE == 0) {
+    if (split_mode && split_parallel(P, T, top, lmap, A, stack_lo, stack_hi)) return;
     if (top[0] <= 32) {  // the whole task fits the register-resident DFS
       run_reg(P, T, top, lmap, A, (RegLevel*)smem, stack_lo, stack_hi, split_mode, smem);
       return;
@@ -1351,6 +1447,50 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
   __syncwarp();
 }
 
+// Children G[a..b) of a published split node (see split_parallel), each followed by its subtree.
+__device__ void run_descriptor(const Params& P, const uint32_t* desc, WarpMem& M, Acc& A) {
+  const uint32_t lane = lane_id();
+  uint32_t* s = pool_ptr(P, desc[1]);
+  const uint32_t a = desc[2], b = desc[3];
+  TaskCtx Tc;
+  Tc.W = s[0];
+  const uint32_t lmap = s[1];
+  Tc.root = s[2];
+  const uint32_t rlen = s[3];
+  Tc.W4 = r4(Tc.W);
+  Tc.E = r4(Tc.W + 2);
+  Tc.map = s + kHdr;
+  Tc.rlist = M.rbuf;
+  Tc.auxref = s[5];
+  Tc.ncw = s[6];
+  Tc.cols = s[7] == 1 ? pool_ptr(P, Tc.auxref - 1) : nullptr;
+  Tc.gx = s[7] == 2 ? pool_ptr(P, Tc.auxref - 1) : nullptr;
+  small_task_init(P, Tc, lmap);
+  uint32_t* node = s + s[4];
+  const uint32_t n = node[0];
+  const uint32_t* dom = node + kHdr + 4 + 4 * n;
+  const uint32_t* G = dom + r4(n);
+  const long long c0 = clock64();
+  for (uint32_t t = a; t < b; t++) {
+    if (M.rbuf) {
+      for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
+      __syncwarp();
+    }
+    uint32_t* ch = M.dyn;
+    if (!fits(P, ch + kHdr + 4 + 4 * n + 4ull * 32 * Tc.W + 16, M.dyn_end)) return;
+    const int r = gen_child_small(P, Tc, node, G[t], ch, A, M.sm_sort, dom);
+    if (r == 2) {
+      if (lane == 0) {
+        ch[3] = 0;
+        ch[4] = kNone;
+      }
+      __syncwarp();
+      run_task<0>(P, Tc, ch, align4(ch + kHdr + 4 + 4 * ch[0]), M.dyn_end, lmap, A, M.sm_sort);
+    }
+  }
+  if (P.per_root_cycles && lane == 0) atomicAdd(P.per_root_cycles + Tc.root, (unsigned long long)(clock64() - c0));
+}
+
 #ifndef GMBE_MIN_BLOCKS
 #define GMBE_MIN_BLOCKS 3  // 80 registers: 24 resident warps per SM (measured best on gh_work)
 #endif
@@ -1379,6 +1519,12 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       PH_START(A);
       __threadfence();  // acquire: the task was written on another SM
       uint32_t* s = pool_ptr(P, task);
+      if (s[0] == kDescMagic) {
+        run_descriptor(P, s, M, A);
+        if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
+        idle = 0;
+        continue;
+      }
       TaskCtx Tc;
       Tc.W = s[0];
       const uint32_t lmap = s[1];
