@@ -114,6 +114,12 @@ typedef struct {
   /* Optional profiling (HOST uint64_t[16]): SM cycles summed over warps per phase (names in the
    * Python binding's PHASES). */
   uint64_t* phase_cycles;
+  /* Optional profiling timeline (DEVICE memory, timeline_cap uint64 words): word 0 = number of
+   * records, then per root / task: [smid<<56 | kind<<48 | root rank, start ns, end ns]
+   * (%globaltimer; kind 0 root, 1 split subtask, 2 split descriptor) -- the active-SM timeline of
+   * PAPER.md Fig 4 / Fig 9. */
+  uint64_t* timeline;
+  uint64_t timeline_cap;
   /* Workspace (0 = auto): words of the per-warp dynamic region (root record, node stack); words
    * of the task pool (split subtasks and shared Γ columns; when it is exhausted work simply stays
    * with the warp that generated it); capacity of the task queue (entries). */

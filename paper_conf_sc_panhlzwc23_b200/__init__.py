@@ -49,7 +49,8 @@ class Opts(ctypes.Structure):
                 ("bound_size", _u32), ("warps_per_sm", _u32), ("part_index", _u32),
                 ("part_count", _u32), ("reserved0", _u32), ("reserved1", _u32),
                 ("out_offsets", _vp), ("out_offsets_cap", _u64), ("out_ids", _vp),
-                ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("phase_cycles", _vp), ("arena_words", _u64),
+                ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("phase_cycles", _vp), ("timeline", _vp), ("timeline_cap", _u64),
+                ("arena_words", _u64),
                 ("pool_words", _u64), ("queue_cap", _u64), ("cuda_stream", _vp)]
 
 
@@ -122,6 +123,7 @@ class Result:
     per_root_count: np.ndarray = field(default=None, repr=False)
     per_root_cycles: np.ndarray = field(default=None, repr=False)
     phase_cycles: dict = field(default=None, repr=False)
+    timeline: np.ndarray = field(default=None, repr=False)
 
 
 def _stream_ptr(stream):
@@ -147,7 +149,7 @@ class Graph:
 
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
-                  per_root=False, root_cycles=False, phases=False, debug=0, arena_words=0, pool_words=0, queue_cap=0, stream=None):
+                  per_root=False, root_cycles=False, phases=False, timeline=0, debug=0, arena_words=0, pool_words=0, queue_cap=0, stream=None):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
@@ -178,6 +180,11 @@ class Graph:
             inf = self.info()
             prcy = np.zeros(max(inf["n_u"] if inf["swapped"] else inf["n_v"], 1), np.uint64)
             o.per_root_cycles = prcy.ctypes.data
+        tl = None
+        if timeline:
+            import torch
+            tl = torch.zeros(1 + 3 * timeline, dtype=torch.int64, device=torch.device("cuda", self.info()["device"]))
+            o.timeline, o.timeline_cap = tl.data_ptr(), 1 + 3 * timeline
         phc = None
         if phases:
             phc = np.zeros(16, np.uint64)
@@ -191,6 +198,10 @@ class Graph:
             res.bicliques = decode_records(offs, ids)
         if root_cycles:
             res.per_root_cycles = prcy
+        if timeline:
+            t = tl.cpu().numpy().view(np.uint64)
+            nrec = min(int(t[0]), timeline)
+            res.timeline = t[1:1 + 3 * nrec].reshape(-1, 3)
         if phases:
             res.phase_cycles = dict(zip(PHASES, phc.tolist()))
         if per_root:

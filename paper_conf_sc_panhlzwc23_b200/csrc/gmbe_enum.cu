@@ -77,7 +77,9 @@ struct Params {
   unsigned long long* per_root;
   unsigned long long* per_root_cycles;
   uint32_t profile;
-  uint32_t debug;  // opts.reserved0 bits (experiments)
+  uint32_t debug;  // opts.reserved0 bits (experiments): 2 = parallel split (split_parallel)
+  unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1]*
+  uint64_t timeline_cap;
 };
 
 struct Acc {
@@ -1143,7 +1145,7 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
   const bool split_mode = heavy(P, top[2], top[0]);
   if (split_mode) A.splits++;
   if constexpr (LPE == 0) {
-    if (split_mode && split_parallel(P, T, top, lmap, A, stack_lo, stack_hi)) return;
+    if (split_mode && (P.debug & 2) && split_parallel(P, T, top, lmap, A, stack_lo, stack_hi)) return;
     if (top[0] <= 32) {  // the whole task fits the register-resident DFS
       run_reg(P, T, top, lmap, A, (RegLevel*)smem, stack_lo, stack_hi, split_mode, smem);
       return;
@@ -1447,6 +1449,28 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
   __syncwarp();
 }
 
+__device__ __forceinline__ unsigned long long globaltimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t v;
+  asm("mov.u32 %0, %%smid;" : "=r"(v));
+  return v;
+}
+// profiling timeline: one record per root / task / descriptor (kind 0 / 1 / 2)
+__device__ void timeline_rec(const Params& P, uint32_t kind, uint32_t root, unsigned long long t0) {
+  if (lane_id() != 0) return;
+  const unsigned long long t1 = globaltimer();
+  const unsigned long long i = atomicAdd(P.timeline, 1ull);
+  if (1 + 3 * (i + 1) > P.timeline_cap) return;
+  unsigned long long* r = P.timeline + 1 + 3 * i;
+  r[0] = ((unsigned long long)smid() << 56) | ((unsigned long long)kind << 48) | root;
+  r[1] = t0;
+  r[2] = t1;
+}
+
 // Children G[a..b) of a published split node (see split_parallel), each followed by its subtree.
 __device__ void run_descriptor(const Params& P, const uint32_t* desc, WarpMem& M, Acc& A) {
   const uint32_t lane = lane_id();
@@ -1520,7 +1544,9 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       __threadfence();  // acquire: the task was written on another SM
       uint32_t* s = pool_ptr(P, task);
       if (s[0] == kDescMagic) {
+        const unsigned long long g0 = P.timeline ? globaltimer() : 0;
         run_descriptor(P, s, M, A);
+        if (P.timeline) timeline_rec(P, 2, 0, g0);
         if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
         idle = 0;
         continue;
@@ -1543,7 +1569,9 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       __syncwarp();
       PH_STOP(A, 15);
       const long long c0 = clock64();
+      const unsigned long long g0 = P.timeline ? globaltimer() : 0;
       dispatch_task(P, Tc, s + s[4], M.dyn, M.dyn_end, lmap, A, M.sm_sort);
+      if (P.timeline) timeline_rec(P, 1, Tc.root, g0);
       if (P.per_root_cycles && lane == 0)
         atomicAdd(P.per_root_cycles + Tc.root, (unsigned long long)(clock64() - c0));
       __syncwarp();
@@ -1562,7 +1590,9 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       if (t < P.n_roots) {
         const uint32_t rk = P.part_index + (P.n_roots - 1 - (uint32_t)t) * P.part_count;
         const long long c0 = clock64();
+        const unsigned long long g0 = P.timeline ? globaltimer() : 0;
         run_root(P, rk, M, A);
+        if (P.timeline) timeline_rec(P, 0, rk, g0);
         if (P.per_root_cycles && lane == 0)
           atomicAdd(P.per_root_cycles + rk, (unsigned long long)(clock64() - c0));
         __syncwarp();
@@ -1817,6 +1847,9 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.per_root_cycles = o.per_root_cycles ? (unsigned long long*)W.per_root_cyc : nullptr;
   P.profile = o.phase_cycles ? 1 : 0;
   P.debug = o.reserved0;
+  P.timeline = (unsigned long long*)o.timeline;
+  P.timeline_cap = o.timeline_cap;
+  if (P.timeline) GMBE_CUDA_TRY(cudaMemsetAsync(P.timeline, 0, 8, s));
 
   Ctrl hc{};
   GMBE_CUDA_TRY(cudaMemcpyAsync(W.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
