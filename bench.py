@@ -29,7 +29,7 @@ CTRL_D2H_BYTES = 1024  # sizeof(Ctrl) read back by gmbe_enumerate (static_assert
 def _args():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default=DEFAULT_CONFIG)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -75,26 +75,23 @@ def _traffic(name):
 
 
 def _cpu_sample(name, budget_s, gold):
-    """Time the oracle (as it stands, 1 thread) on a bounded root shard of the workload."""
+    """Time the oracle (as it stands, 1 thread) on a bounded sample of the workload: root shards
+    i/S (i = 0, 1, ...) of the degree-rank interleave, added until about budget_s of CPU time."""
     import oracle
     from gmbe_inputs import make_config
     nu, nv, e = make_config(name)
     if gold and gold.get("oracle_cpu_seconds"):
         shards = max(1, int(round(gold["oracle_cpu_seconds"] / budget_s)))
     else:
-        shards = 256
-        while True:
-            t = time.time()
-            oracle.oracle_mbe(nu, nv, e, shard=(0, shards))
-            dt = time.time() - t
-            if dt * 8 > budget_s or shards == 1:
-                shards = max(1, int(shards * dt / budget_s)) if dt > 0 else shards
-                break
-            shards //= 8
-    t = time.time()
-    r = oracle.oracle_mbe(nu, nv, e, shard=(0, shards))
-    dt = time.time() - t
-    return r, dt, shards
+        shards = 1024
+    count, dt, taken = 0, 0.0, 0
+    while taken < shards and dt < budget_s:
+        t = time.time()
+        r = oracle.oracle_mbe(nu, nv, e, shard=(taken, shards))
+        dt += time.time() - t
+        count += r.count
+        taken += 1
+    return count, dt, "root shards 0..%d of %d" % (taken - 1, shards)
 
 
 class ClockSampler:
@@ -144,21 +141,22 @@ def run_reference(a):
     gold = _gold(a.config)
     nu, nv, e = make_config(a.config)
     for _ in range(max(0, min(a.warmup, 1))):
-        _cpu_sample(a.config, a.cpu_budget_s / 4, gold)
-    times, counts, shards = [], [], 1
+        _cpu_sample(a.config, 1.0, gold)
+    times, counts, sample = [], [], ""
+    per_step = min(a.cpu_budget_s, 180.0 / max(1, a.steps))  # whole run within a few minutes
     for _ in range(a.steps):
-        r, dt, shards = _cpu_sample(a.config, a.cpu_budget_s, gold)
+        c, dt, sample = _cpu_sample(a.config, per_step, gold)
         times.append(dt)
-        counts.append(r.count)
+        counts.append(c)
     v = sum(counts) / sum(times)
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "bicliques/s",
             "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup,
             "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": a.config, "n_u": nu, "n_v": nv, "m": int(len(e)),
-                       "sample": "root shard 0/%d" % shards},
+                       "sample": sample},
             "cpu_baseline": {"value": v, "unit": "bicliques/s", "cores": 1, "kind": "oracle",
-                             "sample": "oracle single-thread on root shard 0/%d of %s" % (shards, a.config)},
+                             "sample": "oracle single-thread on %s of %s" % (sample, a.config)},
             "e2e": {"value": v, "unit": "bicliques/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -300,10 +298,10 @@ def main():
             "clocks": clocks,
         }
         if ws == 1 and not a.no_cpu_baseline:
-            r, dt, shards = _cpu_sample(a.config, a.cpu_budget_s, gold)
-            line["cpu_baseline"] = {"value": r.count / dt, "unit": "bicliques/s", "cores": 1,
+            c, dt, sample = _cpu_sample(a.config, a.cpu_budget_s, gold)
+            line["cpu_baseline"] = {"value": c / dt, "unit": "bicliques/s", "cores": 1,
                                     "kind": "oracle",
-                                    "sample": "root shard 0/%d (%d bicliques, %.1f s)" % (shards, r.count, dt)}
+                                    "sample": "%s (%d bicliques, %.1f s)" % (sample, c, dt)}
         print(json.dumps(line), flush=True)
     if ws > 1:
         dist.barrier()
