@@ -117,9 +117,11 @@ struct TaskCtx {
   uint32_t root;        // rank of the root vertex
   uint32_t* rlist;      // R-list stack (output only)
   // Γ index of the root (maximality count without binary searches), one of:
-  //   gx  (universe <= 64 bits): [nx, l, -, -] | xrow u64[nx] (row of each 2-hop vertex x over the
-  //        universe) | coff u32[l+1] | cx u32[] (2-hop indices adjacent to universe vertex j)
-  //   cols (larger universes): cols[j*ncw ..] = bitmap of the 2-hop vertices adjacent to vertex j
+  //   gx  (universe <= 64 bits): [nx, l, -, -] | xrow u64[nx] (row of each X2 vertex x over the
+  //        universe) | coff u32[l+1] | cx u32[] (X2 indices adjacent to universe vertex j)
+  //   cols (larger universes): cols[j*ncw ..] = bitmap of the X2 vertices adjacent to vertex j
+  // X2 = the root's 2-hop vertices adjacent to >= 2 universe vertices (the only ones that can cover
+  // an L' with |L'| >= 2).
   // or neither (count Γ by binary search over the adjacency lists).
   const uint32_t* gx;
   const uint32_t* cols;
@@ -129,6 +131,8 @@ struct TaskCtx {
   // small_task_init: Γ-list offsets / lengths and the checksum hashes of the universe vertices
   uint32_t go0, go1, gl0, gl1;
   unsigned long long hu0, hu1;
+  uint32_t nx;                // gx: |X2|; <= 64: the X2 rows are lane-resident in xr0 / xr1
+  unsigned long long xr0, xr1;
   const uint32_t* gxl;  // gx: base of the per-vertex 2-hop lists
 };
 
@@ -746,7 +750,15 @@ __device__ void small_task_init(const Params& P, TaskCtx& T, uint32_t lmap) {
   T.hu0 = lane < lmap ? gmbe_hid(T.map[lane], P.hu_side) : 0ull;
   T.hu1 = lane + 32 < lmap ? gmbe_hid(T.map[lane + 32], P.hu_side) : 0ull;
   T.gxl = nullptr;
+  T.nx = kNone;
+  T.xr0 = T.xr1 = 0;
   if (T.gx) {
+    T.nx = T.gx[0];
+    const unsigned long long* xrow = (const unsigned long long*)(T.gx + 4);
+    if (T.nx <= 64) {
+      if (lane < T.nx) T.xr0 = xrow[lane];
+      if (lane + 32 < T.nx) T.xr1 = xrow[lane + 32];
+    }
     const uint32_t* coff = T.gx + 4 + 2 * T.gx[0];
     const uint32_t l = T.gx[1];
     T.gxl = coff + r4(l + 1);
@@ -764,6 +776,11 @@ __device__ void small_task_init(const Params& P, TaskCtx& T, uint32_t lmap) {
 // maximality with gx and lane-resident list offsets (see gamma_gx_is_r)
 __device__ __forceinline__ bool gamma_gx_small(const TaskCtx& T, unsigned long long lm, uint32_t rlen) {
   const uint32_t lane = lane_id();
+  if (T.nx <= 64) {  // lane-resident X2 rows: |Γ(L')| = 1 + #rows covering L'
+    uint32_t count = 1 + __popc(__ballot_sync(GMBE_FULL, (T.xr0 & lm) == lm));
+    if (T.nx > 32) count += __popc(__ballot_sync(GMBE_FULL, (T.xr1 & lm) == lm));
+    return count == rlen;
+  }
   uint32_t key = 0xffffffffu;
   if ((lm >> lane) & 1ull) key = (T.gl0 << 7) | lane;
   if ((lm >> (lane + 32)) & 1ull) key = min(key, (T.gl1 << 7) | (lane + 32));
@@ -1248,7 +1265,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
   // later-ordered partial neighbours -> C (Alg 3 L5-6); earlier-ordered ones are never candidates
   unsigned long long* sortbuf = (unsigned long long*)align4(M.dyn);
   const uint32_t W = (l + 31) / 32, W4 = r4(W), E = r4(W + 2);
-  uint32_t nC = 0, nR = 0;
+  uint32_t nC = 0, nR = 0, nx2 = 0, sum2 = 0;
   bool skip = false;
   unsigned long long sr = 0;
   const bool sort_fits = fits(P, (uint32_t*)(sortbuf + next_pow2(max(nocc, 1u))) + 64, M.dyn_end);
@@ -1264,6 +1281,9 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
     }
     const bool isR = occ && c == l;
     skip |= isR && v < r;
+    // X2: only 2-hop vertices sharing >= 2 universe vertices can cover an L' with |L'| >= 2
+    nx2 += __popc(__ballot_sync(GMBE_FULL, occ && c >= 2));
+    sum2 += occ && c >= 2 ? c : 0u;
     const bool isC = occ && !isR && v > r;
     if (isR) sr += g.hv[v];
     const uint32_t bR = __ballot_sync(GMBE_FULL, isR);
@@ -1274,12 +1294,14 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
     nC += __popc(bC);
   }
   skip = __any_sync(GMBE_FULL, skip);
+  sum2 = warp_sum(sum2);
   PH_STOP(A, 1);
-  // Γ index over the 2-hop set X (= the occupied table slots; x = position in occ): gx for
-  // universes <= 64 bits, columns otherwise (see TaskCtx)
-  const uint32_t ncw = (nocc + 31) / 32;
+  // Γ index over X2 = {x in the 2-hop set X : |N(x) ∩ L_r| >= 2} (the maximality test of an L' with
+  // |L'| >= 2 only counts vertices covering >= 2 universe vertices; |L'| = 1 uses the degree): gx for
+  // universes <= 64 bits, columns otherwise (see TaskCtx).  x2 = position of x among X2 in occ order.
+  const uint32_t ncw = (nx2 + 31) / 32;
   uint32_t* aux = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
-  const uint64_t aux_words = small ? 4ull + 2ull * nocc + r4(l + 1) + (wedges - l) : (uint64_t)l * ncw;
+  const uint64_t aux_words = small ? 4ull + 2ull * nx2 + r4(l + 1) + sum2 : (uint64_t)l * ncw;
   const bool want_aux = !skip && nC > 0 && aux_words <= P.col_budget;
   const bool want_cols = want_aux && !small;
   uint32_t* cols = aux;
@@ -1302,20 +1324,44 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
     }
     PH_STOP(A, 8);
     if (want_aux && small) {
-      // gx: rows of the 2-hop vertices, and per universe vertex u_j the list of its 2-hop
-      // neighbours (|list_j| = deg(u_j) - 1: every neighbour but v_s lies in X)
+      // gx: rows of the X2 vertices, and per universe vertex u_j the list of its X2 neighbours
       unsigned long long* xrow = (unsigned long long*)(gx + 4);
-      uint32_t* coff = gx + 4 + 2 * nocc;
+      uint32_t* coff = gx + 4 + 2 * nx2;
       uint32_t* cx = coff + r4(l + 1);
       if (lane == 0) {
-        gx[0] = nocc;
+        gx[0] = nx2;
         gx[1] = l;
       }
-      for (uint32_t x = lane; x < nocc; x += 32) xrow[x] = __ldcg(vals + M.occ[x]);
+      uint32_t n2 = 0;
+      for (uint32_t b = 0; b < nocc; b += 32) {
+        const uint32_t x = b + lane;
+        const unsigned long long row = x < nocc ? __ldcg(vals + M.occ[x]) : 0ull;
+        const bool is2 = __popcll(row) >= 2;
+        const uint32_t bal = __ballot_sync(GMBE_FULL, is2);
+        if (is2) xrow[n2 + __popc(bal & lanemask_lt())] = row;
+        n2 += __popc(bal);
+      }
+      __syncwarp();
+      // list lengths: lane j counts universe vertex j (cnt0) and j + 32 (cnt1)
+      uint32_t cnt0 = 0, cnt1 = 0;
+      for (uint32_t b = 0; b < nx2; b += 32) {
+        const unsigned long long row = b + lane < nx2 ? xrow[b + lane] : 0ull;
+        unsigned long long any = ((unsigned long long)__reduce_or_sync(GMBE_FULL, (uint32_t)(row >> 32)) << 32) |
+                                 __reduce_or_sync(GMBE_FULL, (uint32_t)row);
+        while (any) {
+          const uint32_t j = __ffsll(any) - 1;
+          any &= any - 1;
+          const uint32_t c = __popc(__ballot_sync(GMBE_FULL, (row >> j) & 1ull));
+          if (lane == (j & 31)) {
+            if (j < 32) cnt0 += c;
+            else cnt1 += c;
+          }
+        }
+      }
       uint32_t carry = 0, cur0 = 0, cur1 = 0;
       for (uint32_t h = 0; h < 2; h++) {
         const uint32_t j = h * 32 + lane;
-        const uint32_t c = j < l ? g.off_u[Lr[j] + 1] - g.off_u[Lr[j]] - 1 : 0;
+        const uint32_t c = h ? cnt1 : cnt0;
         uint32_t inc = c;
         for (int o = 1; o < 32; o <<= 1) {
           const uint32_t t = __shfl_up_sync(GMBE_FULL, inc, o);
@@ -1329,19 +1375,21 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       }
       if (lane == 0 && l == 64) coff[64] = carry;
       __syncwarp();
-      for (uint32_t b = 0; b < nocc; b += 32) {
+      for (uint32_t b = 0; b < nx2; b += 32) {
         const uint32_t x = b + lane;
-        const unsigned long long row = x < nocc ? xrow[x] : 0ull;
-        for (uint32_t j = 0; j < l; j++) {
+        const unsigned long long row = x < nx2 ? xrow[x] : 0ull;
+        unsigned long long any = ((unsigned long long)__reduce_or_sync(GMBE_FULL, (uint32_t)(row >> 32)) << 32) |
+                                 __reduce_or_sync(GMBE_FULL, (uint32_t)row);
+        while (any) {
+          const uint32_t j = __ffsll(any) - 1;
+          any &= any - 1;
           const bool bit = (row >> j) & 1ull;
           const uint32_t bal = __ballot_sync(GMBE_FULL, bit);
-          if (bal) {
-            const uint32_t base = __shfl_sync(GMBE_FULL, j < 32 ? cur0 : cur1, j & 31);
-            if (bit) cx[base + __popc(bal & lanemask_lt())] = x;
-            if (lane == (j & 31)) {
-              if (j < 32) cur0 += __popc(bal);
-              else cur1 += __popc(bal);
-            }
+          const uint32_t base = __shfl_sync(GMBE_FULL, j < 32 ? cur0 : cur1, j & 31);
+          if (bit) cx[base + __popc(bal & lanemask_lt())] = x;
+          if (lane == (j & 31)) {
+            if (j < 32) cur0 += __popc(bal);
+            else cur1 += __popc(bal);
           }
         }
       }
@@ -1375,10 +1423,19 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
       PH_STOP(A, 10);
       if (!small) {
         // pass 2: candidate rows over L_r, and the Γ columns: table value := x << 32 | C tag + entry
-        for (uint32_t x = lane; x < nocc; x += 32) {
-          const uint32_t s2 = M.occ[x];
-          const unsigned long long v2 = __ldcg(vals + s2);
-          vals[s2] = ((unsigned long long)x << 32) | ((v2 & kCTag) ? (0x80000000ull | (uint32_t)v2) : 0ull);
+        // table value := (x2 + 1) << 32 (0: not in X2) | C tag + entry
+        uint32_t n2 = 0;
+        for (uint32_t b = 0; b < nocc; b += 32) {
+          const uint32_t x = b + lane;
+          const uint32_t s2 = x < nocc ? M.occ[x] : 0u;
+          const unsigned long long v2 = x < nocc ? __ldcg(vals + s2) : 0ull;
+          const bool isc = (v2 & kCTag) != 0;
+          const uint32_t k = isc ? ent[(size_t)(uint32_t)(v2 & 0x7fffffffull) * E + W + 1] : (uint32_t)v2;
+          const bool is2 = x < nocc && k >= 2;
+          const uint32_t bal = __ballot_sync(GMBE_FULL, is2);
+          const unsigned long long x2 = is2 ? (unsigned long long)(n2 + __popc(bal & lanemask_lt()) + 1) : 0ull;
+          n2 += __popc(bal);
+          if (x < nocc) vals[s2] = (x2 << 32) | (isc ? (0x80000000ull | (uint32_t)v2) : 0ull);
         }
         if (want_cols)
           for (uint64_t j = lane; j < (uint64_t)l * ncw; j += 32) cols[j] = 0;
@@ -1388,7 +1445,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
             const uint32_t h = ht_find(keys, shift, mask, v);
             const unsigned long long x = __ldcg(vals + h);
             const uint32_t xi = (uint32_t)(x >> 32);
-            if (want_cols) atomicOr(cols + (size_t)i * ncw + (xi >> 5), 1u << (xi & 31));
+            if (want_cols && xi) atomicOr(cols + (size_t)i * ncw + ((xi - 1) >> 5), 1u << ((xi - 1) & 31));
             if (x & 0x80000000ull) atomicOr(ent + (size_t)(x & 0x7fffffffull) * E + (i >> 5), 1u << (i & 31));
           }
         });
