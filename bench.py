@@ -23,7 +23,7 @@ sys.path.insert(0, ROOT)
 
 DEFAULT_CONFIG = "gh_work"
 METRIC = "maximal bicliques/sec (Github-shaped)"
-CTRL_D2H_BYTES = 1024  # sizeof(Ctrl) read back by gmbe_enumerate (static_assert in gmbe_enum.cu)
+CTRL_BYTES = 1152  # sizeof(Ctrl): written and read back by gmbe_enumerate (static_assert in gmbe_enum.cu)
 
 
 def _args():
@@ -286,7 +286,7 @@ def main():
             "kernel_ms": k_rank,
             "host_wall_ms": {k: round(sum(v[-a.steps:]) / max(1, len(v[-a.steps:])), 3) for k, v in host_ms.items()},
             "e2e": {"value": count / (t_e2e * 1e-3), "unit": "bicliques/s",
-                    "h2d_bytes_per_step": int(m * 8), "d2h_bytes_per_step": CTRL_D2H_BYTES},
+                    "h2d_bytes_per_step": int(m * 8) + CTRL_BYTES, "d2h_bytes_per_step": CTRL_BYTES},
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "kernel": "k_enum", "achieved": achieved, "peak": peak,
                          "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak,
@@ -294,7 +294,7 @@ def main():
                          "algo_bytes_per_launch": abytes, "algo_bytes_definition": adef,
                          "algo_bytes_cand": rc.algo_bytes_cand},
             "work": {"nodes": rc.nodes, "nonmax": rc.nonmax, "roots_run": rc.roots_run,
-                     "splits": rc.splits, "tasks": rc.tasks},
+                     "splits": rc.splits, "tasks": rc.tasks, "donations": rc.donations},
             "clocks": clocks,
         }
         if ws == 1 and not a.no_cpu_baseline:

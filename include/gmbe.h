@@ -115,9 +115,9 @@ typedef struct {
    * Python binding's PHASES). */
   uint64_t* phase_cycles;
   /* Optional profiling timeline (DEVICE memory, timeline_cap uint64 words): word 0 = number of
-   * records, then per root / task: [smid<<56 | kind<<48 | root rank, start ns, end ns]
-   * (%globaltimer; kind 0 root, 1 split subtask, 2 split descriptor) -- the active-SM timeline of
-   * PAPER.md Fig 4 / Fig 9. */
+   * records, then per root / task: [smid<<56 | kind<<48 | root rank, start ns, end ns,
+   * nodes<<32 | min(|L_top|,65535)<<16 | min(|C_top|,65535)] (%globaltimer; kind 0 root, 1 split
+   * subtask, 2 split descriptor) -- the active-SM timeline of PAPER.md Fig 4 / Fig 9. */
   uint64_t* timeline;
   uint64_t timeline_cap;
   /* Workspace (0 = auto): words of the per-warp dynamic region (root record, node stack); words
@@ -141,6 +141,7 @@ typedef struct {
                                (the Q term is not computed on the GPU) */
   uint64_t splits;        /* nodes expanded in split mode */
   uint64_t tasks;         /* subtasks enqueued */
+  uint64_t donations;     /* subtasks donated to idle warps (dynamic load balancing) */
   double kernel_ms;       /* device time of the enumeration kernel (CUDA events) */
 } gmbe_result;
 

@@ -57,7 +57,7 @@ class Opts(ctypes.Structure):
 class CResult(ctypes.Structure):
     _fields_ = [(n, _u64) for n in ("count", "checksum", "n_written", "truncated", "roots_run",
                                      "nodes", "nonmax", "algo_bytes_cand", "splits",
-                                     "tasks")] + [("kernel_ms", ctypes.c_double)]
+                                     "tasks", "donations")] + [("kernel_ms", ctypes.c_double)]
 
 
 _lib.gmbe_load_bipartite.argtypes = [_u32, _u32, _vp, _u64, ctypes.POINTER(LoadOpts), ctypes.POINTER(_vp)]
@@ -118,6 +118,7 @@ class Result:
     algo_bytes_cand: int
     splits: int
     tasks: int
+    donations: int
     kernel_ms: float
     bicliques: list = field(default=None, repr=False)
     per_root_count: np.ndarray = field(default=None, repr=False)
@@ -183,8 +184,8 @@ class Graph:
         tl = None
         if timeline:
             import torch
-            tl = torch.zeros(1 + 3 * timeline, dtype=torch.int64, device=torch.device("cuda", self.info()["device"]))
-            o.timeline, o.timeline_cap = tl.data_ptr(), 1 + 3 * timeline
+            tl = torch.zeros(1 + 4 * timeline, dtype=torch.int64, device=torch.device("cuda", self.info()["device"]))
+            o.timeline, o.timeline_cap = tl.data_ptr(), 1 + 4 * timeline
         phc = None
         if phases:
             phc = np.zeros(16, np.uint64)
@@ -201,7 +202,7 @@ class Graph:
         if timeline:
             t = tl.cpu().numpy().view(np.uint64)
             nrec = min(int(t[0]), timeline)
-            res.timeline = t[1:1 + 3 * nrec].reshape(-1, 3)
+            res.timeline = t[1:1 + 4 * nrec].reshape(-1, 4)
         if phases:
             res.phase_cycles = dict(zip(PHASES, phc.tolist()))
         if per_root:

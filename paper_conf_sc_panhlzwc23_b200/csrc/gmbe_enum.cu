@@ -43,13 +43,14 @@ struct alignas(128) Line {
 };
 struct Ctrl {
   Line root_cursor, q_head, q_tail, q_avail, pending, pool_next;
-  unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
+  Line hungry;  // warps idle-waiting for work (all roots issued, queue empty): triggers donation
+  unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks, donations;
   unsigned long long out_rec, out_ids;
   unsigned long long phase[16];
   unsigned int truncated, error;
 };
 
-static_assert(sizeof(Ctrl) == 1024, "bench.py reports sizeof(Ctrl) as the per-step D2H bytes");
+static_assert(sizeof(Ctrl) == 1152, "bench.py reports sizeof(Ctrl) as the per-step D2H / H2D control bytes");
 
 enum : unsigned int { kErrArena = 1 };
 
@@ -77,13 +78,14 @@ struct Params {
   unsigned long long* per_root;
   unsigned long long* per_root_cycles;
   uint32_t profile;
-  uint32_t debug;  // opts.reserved0 bits (experiments): 2 = parallel split (split_parallel)
-  unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1]*
+  uint32_t debug;  // opts.reserved0 bits (experiments): 2 = parallel split (split_parallel), 4 = no donation
+  uint32_t donate;  // dynamic donation to idle warps (donate_reg)
+  unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1, info]*
   uint64_t timeline_cap;
 };
 
 struct Acc {
-  unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks;
+  unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks, donations;
 #ifdef GMBE_PROFILE
   unsigned long long ph[16];  // profiling build only: SM cycles per phase (opts.phase_cycles)
   long long t0;
@@ -936,6 +938,73 @@ __device__ __forceinline__ unsigned long long shfl64(unsigned long long x, uint3
   const uint32_t hi = __shfl_sync(GMBE_FULL, (uint32_t)(x >> 32), src);
   return ((unsigned long long)hi << 32) | lo;
 }
+// Dynamic donation (beyond the paper's static estimate): while warps are idle-waiting
+// (ctrl.hungry > 0), a warp deep in a subtree hands the remaining children of its shallowest
+// unfinished level to the queue as a subtask.  The subtask's node is (L_k, R_k, remaining
+// candidates of level k); its children, their later sets and their Thm 4.1 marks are exactly the
+// ones the donor would have generated, so the tree and every counter are unchanged.
+__device__ __forceinline__ bool hungry(const Params& P) {
+  uint32_t h = 0;
+  if (lane_id() == 0) h = ld_volatile(&P.ctrl->hungry.v) != 0;
+  return __shfl_sync(GMBE_FULL, h, 0) != 0;
+}
+#ifndef GMBE_DONATE
+#define GMBE_DONATE 2  // 0: compiled out; 1: checked every 32 nodes; 2: checked every 8th push
+#endif
+#ifndef GMBE_DONATE_INLINE
+#define GMBE_DONATE_INLINE 1
+#endif
+#if GMBE_DONATE_INLINE
+#define GMBE_DONATE_ATTR __forceinline__
+#else
+#define GMBE_DONATE_ATTR __noinline__
+#endif
+__device__ GMBE_DONATE_ATTR bool donate_reg(const Params& P, const TaskCtx& T, uint32_t lmap, Acc& A, RegLevel* st, uint32_t d,
+                           unsigned long long row, uint32_t id, uint32_t* scratch, const uint32_t* scratch_end) {
+  const uint32_t lane = lane_id();
+  const bool w2 = T.W == 2;
+  uint32_t av = 0;
+  if (lane < d) {
+    const uint32_t nx = st[lane].next;
+    av = nx >= 32 ? 0u : (st[lane].C & ~((1u << nx) - 1u));
+  }
+  const uint32_t b = __ballot_sync(GMBE_FULL, av != 0);
+  if (!b) return false;
+  const uint32_t k = __ffs(b) - 1;
+  av = __shfl_sync(GMBE_FULL, av, k);
+  const unsigned long long Lk = st[k].L, SRk = st[k].SR;
+  const uint32_t rk = st[k].rlen, n = __popc(av);
+  const uint32_t words = kHdr + 4 + 4 * n;
+  if (scratch + words > scratch_end) return false;
+  uint4* ce = (uint4*)(scratch + kHdr + 4);
+  if ((av >> lane) & 1u) {
+    const unsigned long long xr = row & Lk;
+    const uint32_t kc = __popcll(xr);
+    ce[__popc(av & lanemask_lt())] = w2 ? make_uint4((uint32_t)xr, (uint32_t)(xr >> 32), id, kc)
+                                        : make_uint4((uint32_t)xr, id, kc, 0);
+  }
+  if (lane == 0) {
+    scratch[0] = n;
+    scratch[1] = 0;
+    scratch[2] = __popcll(Lk);
+    scratch[3] = 0;
+    scratch[4] = kNone;
+    scratch[5] = rk;
+    scratch[6] = (uint32_t)SRk;
+    scratch[7] = (uint32_t)(SRk >> 32);
+    scratch[kHdr] = (uint32_t)Lk;
+    scratch[kHdr + 1] = (uint32_t)(Lk >> 32);
+    scratch[kHdr + 2] = 0;
+    scratch[kHdr + 3] = 0;
+  }
+  __syncwarp();
+  if (!task_publish(P, T, lmap, T.rlist ? rk : 0, scratch, words, A)) return false;
+  if (lane == 0) st[k].next = 32;  // the donated children are no longer this warp's
+  __syncwarp();
+  A.donations++;
+  return true;
+}
+
 __device__ void run_reg(const Params& P, const TaskCtx& T, const uint32_t* rec, uint32_t lmap, Acc& A,
                         RegLevel* st, uint32_t* scratch, const uint32_t* scratch_end, bool split_top,
                         unsigned long long* smem) {
@@ -954,7 +1023,13 @@ __device__ void run_reg(const Params& P, const TaskCtx& T, const uint32_t* rec, 
   unsigned long long SR = ((unsigned long long)rec[7] << 32) | rec[6];
   uint32_t C = nC >= 32 ? GMBE_FULL : ((1u << nC) - 1u), next = 0, rlen = rec[5];
   int d = 0;
+#if GMBE_DONATE
+  uint32_t tick = 0;
+#endif
   while (true) {
+#if GMBE_DONATE == 1
+    if (d > 0 && (++tick & 31) == 0 && hungry(P)) donate_reg(P, T, lmap, A, st, d, row, id, scratch, scratch_end);
+#endif
     const uint32_t avail = next >= 32 ? 0u : (C & ~((1u << next) - 1u));
     if (!avail) {  // pop (Alg 2 L4)
       if (d == 0) break;
@@ -1046,6 +1121,9 @@ __device__ void run_reg(const Params& P, const TaskCtx& T, const uint32_t* rec, 
       }
     }
     // push (Alg 2 L16)
+#if GMBE_DONATE == 2
+    if (d > 0 && (++tick & 7) == 0 && hungry(P)) donate_reg(P, T, lmap, A, st, d, row, id, scratch, scratch_end);
+#endif
     if (lane == 0) {
       st[d].L = L;
       st[d].SR = SR;
@@ -1517,15 +1595,21 @@ __device__ __forceinline__ uint32_t smid() {
   return v;
 }
 // profiling timeline: one record per root / task / descriptor (kind 0 / 1 / 2)
-__device__ void timeline_rec(const Params& P, uint32_t kind, uint32_t root, unsigned long long t0) {
+// info = nodes generated by the record << 32 | min(|L_top|, 65535) << 16 | min(|C_top|, 65535)
+__device__ void timeline_rec(const Params& P, uint32_t kind, uint32_t root, unsigned long long t0,
+                             unsigned long long info) {
   if (lane_id() != 0) return;
   const unsigned long long t1 = globaltimer();
   const unsigned long long i = atomicAdd(P.timeline, 1ull);
-  if (1 + 3 * (i + 1) > P.timeline_cap) return;
-  unsigned long long* r = P.timeline + 1 + 3 * i;
+  if (1 + 4 * (i + 1) > P.timeline_cap) return;
+  unsigned long long* r = P.timeline + 1 + 4 * i;
   r[0] = ((unsigned long long)smid() << 56) | ((unsigned long long)kind << 48) | root;
   r[1] = t0;
   r[2] = t1;
+  r[3] = info;
+}
+__device__ __forceinline__ unsigned long long tl_info(unsigned long long nodes, uint32_t l, uint32_t c) {
+  return (nodes << 32) | ((unsigned long long)min(l, 65535u) << 16) | min(c, 65535u);
 }
 
 // Children G[a..b) of a published split node (see split_parallel), each followed by its subtree.
@@ -1589,7 +1673,7 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
   M.rbuf = P.rbuf ? P.rbuf + (uint64_t)gw * P.rbuf_words : nullptr;
   M.sm_sort = s_sort[threadIdx.x >> 5];
   Acc A = {};
-  bool roots_done = false;
+  bool roots_done = false, is_hungry = false;
   uint32_t idle = 0;
   while (true) {
     // 1. split subtasks first (Alg 4 L3-4)
@@ -1597,13 +1681,17 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
     if (lane == 0) task = queue_pop(P);
     task = __shfl_sync(GMBE_FULL, task, 0);
     if (task != kNone) {
+      if (is_hungry) {
+        if (lane == 0) atomicAdd(&P.ctrl->hungry.v, ~0ull);
+        is_hungry = false;
+      }
       PH_START(A);
       __threadfence();  // acquire: the task was written on another SM
       uint32_t* s = pool_ptr(P, task);
       if (s[0] == kDescMagic) {
-        const unsigned long long g0 = P.timeline ? globaltimer() : 0;
+        const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
         run_descriptor(P, s, M, A);
-        if (P.timeline) timeline_rec(P, 2, 0, g0);
+        if (P.timeline) timeline_rec(P, 2, 0, g0, tl_info(A.nodes - n0, 0, s[3] - s[2]));
         if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
         idle = 0;
         continue;
@@ -1626,9 +1714,10 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       __syncwarp();
       PH_STOP(A, 15);
       const long long c0 = clock64();
-      const unsigned long long g0 = P.timeline ? globaltimer() : 0;
+      const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
+      const uint32_t tl_l = s[s[4] + 2], tl_c = s[s[4]];
       dispatch_task(P, Tc, s + s[4], M.dyn, M.dyn_end, lmap, A, M.sm_sort);
-      if (P.timeline) timeline_rec(P, 1, Tc.root, g0);
+      if (P.timeline) timeline_rec(P, 1, Tc.root, g0, tl_info(A.nodes - n0, tl_l, tl_c));
       if (P.per_root_cycles && lane == 0)
         atomicAdd(P.per_root_cycles + Tc.root, (unsigned long long)(clock64() - c0));
       __syncwarp();
@@ -1647,9 +1736,10 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       if (t < P.n_roots) {
         const uint32_t rk = P.part_index + (P.n_roots - 1 - (uint32_t)t) * P.part_count;
         const long long c0 = clock64();
-        const unsigned long long g0 = P.timeline ? globaltimer() : 0;
+        const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
         run_root(P, rk, M, A);
-        if (P.timeline) timeline_rec(P, 0, rk, g0);
+        if (P.timeline)
+          timeline_rec(P, 0, rk, g0, tl_info(A.nodes - n0, P.g.off_v[rk + 1] - P.g.off_v[rk], 0));
         if (P.per_root_cycles && lane == 0)
           atomicAdd(P.per_root_cycles + rk, (unsigned long long)(clock64() - c0));
         __syncwarp();
@@ -1665,6 +1755,10 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
     if (lane == 0) pend = ld_volatile(&P.ctrl->pending.v);
     pend = __shfl_sync(GMBE_FULL, pend, 0);
     if (pend == 0) break;
+    if (!is_hungry && P.donate) {  // ask the working warps to donate (see donate_reg)
+      if (lane == 0) atomicAdd(&P.ctrl->hungry.v, 1ull);
+      is_hungry = true;
+    }
     __nanosleep(idle < 4 ? 500 : (idle < 16 ? 2000 : 8000));  // exponential-ish backoff
     idle++;
   }
@@ -1678,6 +1772,7 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
     atomicAdd(&c->abytes, A.abytes);
     atomicAdd(&c->splits, A.splits);
     atomicAdd(&c->tasks, A.tasks);
+    atomicAdd(&c->donations, A.donations);
 #ifdef GMBE_PROFILE
     if (P.profile)
       for (int k = 0; k < 16; k++) atomicAdd(&c->phase[k], A.ph[k]);
@@ -1904,6 +1999,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.per_root_cycles = o.per_root_cycles ? (unsigned long long*)W.per_root_cyc : nullptr;
   P.profile = o.phase_cycles ? 1 : 0;
   P.debug = o.reserved0;
+  P.donate = (o.reserved0 & 4) ? 0 : 1;
   P.timeline = (unsigned long long*)o.timeline;
   P.timeline_cap = o.timeline_cap;
   if (P.timeline) GMBE_CUDA_TRY(cudaMemsetAsync(P.timeline, 0, 8, s));
@@ -1951,6 +2047,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   out->algo_bytes_cand = hc.abytes;
   out->splits = hc.splits;
   out->tasks = hc.tasks;
+  out->donations = hc.donations;
   out->kernel_ms = ms;
   if (o.phase_cycles)
     for (int k = 0; k < 16; k++) o.phase_cycles[k] = hc.phase[k];

@@ -9,16 +9,18 @@ import paper_conf_sc_panhlzwc23_b200 as gmbe  # noqa: E402
 from gmbe_inputs import make_config  # noqa: E402
 
 name = sys.argv[1]
+kw = dict(a.split("=") for a in sys.argv[2:] if "=" in a)
+kw = {k: int(v) for k, v in kw.items()}
 nu, nv, e = make_config(name)
 g = gmbe.load(nu, nv, e)
-full = g.enumerate()
-full = g.enumerate()
-out = {"config": name, "n1_ms": full.kernel_ms, "count": full.count}
-for n in map(int, sys.argv[2:]):
+full = g.enumerate(**kw)
+full = g.enumerate(**kw)
+out = {"config": name, "opts": kw, "n1_ms": full.kernel_ms, "count": full.count}
+for n in [int(a) for a in sys.argv[2:] if "=" not in a]:
     ts, cnt = [], 0
     for i in range(n):
-        g.enumerate(part=(i, n))
-        r = g.enumerate(part=(i, n))
+        g.enumerate(part=(i, n), **kw)
+        r = g.enumerate(part=(i, n), **kw)
         ts.append(r.kernel_ms)
         cnt += r.count
     assert cnt == full.count

@@ -19,5 +19,5 @@ for spec in sys.argv[2:]:
     for _ in range(3):
         r = g.enumerate(**kw)
         ts.append(r.kernel_ms)
-    print("%-50s count %d  kernel ms %s  splits %d tasks %d" % (spec, r.count, " ".join("%.1f" % t for t in ts),
-                                                             r.splits, r.tasks), flush=True)
+    print("%-40s count %d  kernel ms %s  splits %d tasks %d donations %d" % (
+        spec, r.count, " ".join("%.1f" % t for t in ts), r.splits, r.tasks, r.donations), flush=True)

@@ -35,7 +35,9 @@ dur = t1 - t0
 order = np.argsort(-dur)[:10]
 out = dict(config=name, kernel_ms=r.kernel_ms, records=len(t), span_us=float(end),
            busy_warps_per_bin=[round(float(x), 1) for x in busy],
-           longest=[dict(kind=int(kind[i]), sm=int(sm[i]), start_us=round(float(t0[i]), 1),
-                         dur_us=round(float(dur[i]), 1)) for i in order],
+           longest=[dict(kind=int(kind[i]), sm=int(sm[i]), root=int(t[i, 0] & 0xFFFFFFFFFFFF),
+                         start_us=round(float(t0[i]), 1), dur_us=round(float(dur[i]), 1),
+                         nodes=int(t[i, 3] >> 32), l_top=int((t[i, 3] >> 16) & 0xFFFF), c_top=int(t[i, 3] & 0xFFFF))
+                    for i in order],
            last_end_by_kind={int(k): round(float(t1[kind == k].max()), 1) for k in np.unique(kind)})
 print(json.dumps(out))
