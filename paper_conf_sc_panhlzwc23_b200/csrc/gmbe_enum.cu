@@ -78,7 +78,7 @@ struct Params {
   unsigned long long* per_root;
   unsigned long long* per_root_cycles;
   uint32_t profile;
-  uint32_t debug;  // opts.reserved0 bits (experiments): 2 = parallel split (split_parallel), 4 = no donation
+  uint32_t debug;  // opts.reserved0 bits (tests / experiments): 4 = no donation, 8 = donate whenever possible
   uint32_t donate;  // dynamic donation to idle warps (donate_reg)
   unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1, info]*
   uint64_t timeline_cap;
@@ -139,6 +139,25 @@ struct TaskCtx {
 };
 
 // per-warp memory
+// Code size: k_enum's hot paths are inlined; per-root / per-task entry points can be kept out of
+// line (GMBE_NI_* = 1) so the instruction footprint stays within the SM's instruction caches.
+#ifndef GMBE_NI_ROOT
+#define GMBE_NI_ROOT 0
+#endif
+#ifndef GMBE_NI_DISPATCH
+#define GMBE_NI_DISPATCH 0
+#endif
+#ifndef GMBE_NI_REG
+#define GMBE_NI_REG 0
+#endif
+#ifndef GMBE_NI_GAMMA
+#define GMBE_NI_GAMMA 0
+#endif
+#define GMBE_NI_IF(x) GMBE_NI_IF_(x)
+#define GMBE_NI_IF_(x) GMBE_NI_IF_##x
+#define GMBE_NI_IF_0
+#define GMBE_NI_IF_1 __noinline__
+
 struct WarpMem {
   uint32_t* keys;               // clean hash table keys (EMPTY)
   unsigned long long* vals;     // clean hash table values (0)
@@ -474,7 +493,7 @@ __device__ __forceinline__ bool bsearch_rank(const uint32_t* a, uint32_t n, uint
 // Count over N(u*) for the lowest-degree u* ∈ L', testing the other members of L' in increasing
 // degree order (early exit).  L' = the lc set bits of lmask (W words) over map.
 // scratch: room for next_pow2(lc) 64-bit keys (used when lc > 32).
-__device__ bool gamma_is_r(const Params& P, const uint32_t* lmask, uint32_t W, const uint32_t* map, uint32_t lc,
+__device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_is_r(const Params& P, const uint32_t* lmask, uint32_t W, const uint32_t* map, uint32_t lc,
                            uint32_t rlen, unsigned long long* scratch, unsigned long long* smem) {
   const uint32_t lane = lane_id();
   const DevGraph& g = P.g;
@@ -544,7 +563,7 @@ __device__ bool gamma_is_r(const Params& P, const uint32_t* lmask, uint32_t W, c
 
 // Alg 2 L14 with the root's Γ columns: every v ∈ Γ(L') other than v_s lies in the root's 2-hop set
 // X, so |Γ(L')| = 1 + popc(AND_{j ∈ L'} col_j); maximal iff that equals |R'|.
-__device__ bool gamma_cols_is_r(const TaskCtx& T, const uint32_t* lmask, uint32_t W, uint32_t rlen) {
+__device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_cols_is_r(const TaskCtx& T, const uint32_t* lmask, uint32_t W, uint32_t rlen) {
   const uint32_t lane = lane_id();
   const uint32_t need = rlen - 1;  // dominators in X that are already in R'
   uint32_t count = 0;
@@ -804,11 +823,8 @@ __device__ __forceinline__ bool gamma_gx_small(const TaskCtx& T, unsigned long l
 
 // gen_child for W <= 2: one lane per candidate entry, loaded as one 16-byte vector
 // ({row, id, k, -} for W = 1, {row_lo, row_hi, id, k} for W = 2); L' and rows as 64-bit masks.
-// dom != null: `par` is a published split node (read-only, shared by several warps) and the later
-// candidates of child i are {k > i : dom[k] >= i} -- the Thm 4.1 marks of the earlier siblings,
-// precomputed by split_parallel -- so no compaction / marking happens here.
 __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par, uint32_t i, uint32_t* ch, Acc& A,
-                               unsigned long long* smem, const uint32_t* dom = nullptr) {
+                               unsigned long long* smem) {
   const uint32_t lane = lane_id();
   const bool w2 = T.W == 2;
   const uint32_t nC = par[0];
@@ -832,7 +848,7 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
   const uint32_t rl_base = par[5] + 1;
   for (uint32_t base = i + 1; base < nC; base += 32) {
     const uint32_t j = base + lane;
-    const bool in = j < nC && (!dom || dom[j] >= i);
+    const bool in = j < nC;
     uint4 x = make_uint4(0, 0, 0, 0);
     if (in) x = pent[j];
     const unsigned long long row = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
@@ -853,16 +869,14 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
       cent[nCc + __popc(bc & lanemask_lt())] =
           w2 ? make_uint4((uint32_t)xr, (uint32_t)(xr >> 32), id, cnt) : make_uint4((uint32_t)xr, id, cnt, 0);
     nCc += __popc(bc);
-    if (!dom) {
-      const uint32_t bs = __ballot_sync(GMBE_FULL, surv);
-      const uint32_t spos = i + 1 + nsurv + __popc(bs & lanemask_lt());
-      nsurv += __popc(bs);
-      __syncwarp();
-      if (surv && spos != j) pent[spos] = x;
-      __syncwarp();
-    }
+    const uint32_t bs = __ballot_sync(GMBE_FULL, surv);
+    const uint32_t spos = i + 1 + nsurv + __popc(bs & lanemask_lt());
+    nsurv += __popc(bs);
+    __syncwarp();
+    if (surv && spos != j) pent[spos] = x;
+    __syncwarp();
   }
-  if (lane == 0 && !dom) par[0] = i + 1 + nsurv;
+  if (lane == 0) par[0] = i + 1 + nsurv;
   A.nodes++;
   A.abytes += 4ull * (lc + warp_sum64r(later_k));
   const uint32_t rlen = par[5] + 1 + r_abs;
@@ -945,7 +959,7 @@ __device__ __forceinline__ unsigned long long shfl64(unsigned long long x, uint3
 // ones the donor would have generated, so the tree and every counter are unchanged.
 __device__ __forceinline__ bool hungry(const Params& P) {
   uint32_t h = 0;
-  if (lane_id() == 0) h = ld_volatile(&P.ctrl->hungry.v) != 0;
+  if (lane_id() == 0) h = P.donate && ((P.debug & 8) || ld_volatile(&P.ctrl->hungry.v) != 0);
   return __shfl_sync(GMBE_FULL, h, 0) != 0;
 }
 #ifndef GMBE_DONATE
@@ -1005,7 +1019,7 @@ __device__ GMBE_DONATE_ATTR bool donate_reg(const Params& P, const TaskCtx& T, u
   return true;
 }
 
-__device__ void run_reg(const Params& P, const TaskCtx& T, const uint32_t* rec, uint32_t lmap, Acc& A,
+__device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& T, const uint32_t* rec, uint32_t lmap, Acc& A,
                         RegLevel* st, uint32_t* scratch, const uint32_t* scratch_end, bool split_top,
                         unsigned long long* smem) {
   const uint32_t lane = lane_id();
@@ -1141,96 +1155,6 @@ __device__ void run_reg(const Params& P, const TaskCtx& T, const uint32_t* rec, 
   }
 }
 
-// ---------------------------------------------------------------- parallel split (a7)
-// Thm 4.1 at a node prunes candidate c for the later siblings of child i iff k'(c) = k(c), i.e.
-// row(c) ⊆ row(c_i).  Subset domination is transitive, so c_k is pruned before its own turn iff some
-// earlier candidate's row contains row(c_k), and the earliest such one, dom(k), is itself generated.
-// Hence: children = G = {j : dom(j) undefined}, and the later set of child j is {k > j : dom(k) >= j}.
-// split_parallel computes dom / G for a heavy task top (universe <= 64 bits), publishes the node once
-// (read-only) and enqueues range descriptors over G, so sibling children are generated by different
-// warps instead of one sequential loop (the tree, and every counter, is unchanged).
-constexpr uint32_t kDescMagic = 0xFFFFFFF0u;
-constexpr uint32_t kDescChildren = 4;  // children per descriptor
-__device__ bool split_parallel(const Params& P, const TaskCtx& T, const uint32_t* top, uint32_t lmap, Acc& A,
-                               uint32_t* scratch, const uint32_t* scratch_end) {
-  const uint32_t lane = lane_id();
-  const bool w2 = T.W == 2;
-  const uint32_t n = top[0];
-  const uint32_t words = kHdr + 4 + 4 * n;  // node record (W <= 2: 16-byte entries)
-  uint32_t* dom = scratch;
-  uint32_t* G = dom + r4(n);
-  if (G + r4(n) + 64 > scratch_end || !queue_room(P)) return false;
-  const uint4* ent = (const uint4*)(top + kHdr + 4);
-  uint32_t ng = 0;
-  for (uint32_t kb = 0; kb < n; kb += 32) {
-    const uint32_t k = kb + lane;
-    unsigned long long rk = 0;
-    if (k < n) {
-      const uint4 x = ent[k];
-      rk = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
-    }
-    uint32_t d = k < n ? kNone : 0u;
-    // dominators among the generated candidates of earlier chunks
-    for (uint32_t t = 0; t < ng && __any_sync(GMBE_FULL, d == kNone); t++) {
-      const uint32_t gi = G[t];
-      const uint4 x = ent[gi];
-      const unsigned long long ri = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
-      if (d == kNone && (ri & rk) == rk) d = gi;
-    }
-    // within the chunk, in order
-    for (uint32_t t = 0; t < 32 && kb + t < n; t++) {
-      const bool gen_t = __shfl_sync(GMBE_FULL, d, t) == kNone;
-      if (gen_t) {
-        const unsigned long long rt = shfl64(rk, t);
-        if (lane > t && d == kNone && (rt & rk) == rk) d = kb + t;
-      }
-    }
-    if (k < n) dom[k] = d;
-    const uint32_t bg = __ballot_sync(GMBE_FULL, k < n && d == kNone);
-    if (k < n && d == kNone) G[ng + __popc(bg & lanemask_lt())] = k;
-    ng += __popc(bg);
-    __syncwarp();
-  }
-  // publish: task record (map | R list | node | dom | G) + descriptors over G
-  const uint32_t rlen = T.rlist ? top[5] : 0;
-  const uint32_t node_off = task_node_off(lmap, rlen);
-  const uint32_t total = node_off + words + r4(n) + r4(ng);
-  const uint32_t nd = (ng + kDescChildren - 1) / kDescChildren;
-  const uint32_t off16 = pool_alloc(P, r4(total) + 4 * nd);
-  if (off16 == kNone) return false;
-  uint32_t* s = pool_ptr(P, off16);
-  for (uint32_t j = lane; j < lmap; j += 32) s[kHdr + j] = T.map[j];
-  if (T.rlist)
-    for (uint32_t j = lane; j < rlen; j += 32) s[kHdr + r4(lmap) + j] = T.rlist[j];
-  for (uint32_t j = lane; j < words; j += 32) s[node_off + j] = top[j];
-  uint32_t* sd = s + node_off + words;
-  for (uint32_t j = lane; j < n; j += 32) sd[j] = dom[j];
-  for (uint32_t j = lane; j < ng; j += 32) sd[r4(n) + j] = G[j];
-  uint32_t* desc = s + r4(total);
-  for (uint32_t t = lane; t < nd; t += 32) {
-    desc[4 * t] = kDescMagic;
-    desc[4 * t + 1] = off16;
-    desc[4 * t + 2] = t * kDescChildren;
-    desc[4 * t + 3] = min(ng, (t + 1) * kDescChildren);
-  }
-  if (lane == 0) {
-    s[0] = T.W;
-    s[1] = lmap;
-    s[2] = T.root;
-    s[3] = rlen;
-    s[4] = node_off;
-    s[5] = T.auxref;
-    s[6] = T.ncw;
-    s[7] = T.auxref ? (T.gx ? 2u : 1u) : 0u;
-  }
-  A.tasks += nd;
-  __threadfence();
-  __syncwarp();
-  const uint32_t desc16 = off16 + r4(total) / 4;
-  for (uint32_t t = lane; t < nd; t += 32) queue_push(P, desc16 + t);
-  return true;
-}
-
 template <int LPE>
 __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint32_t* stack_lo, uint32_t* stack_hi,
                          uint32_t lmap, Acc& A, unsigned long long* smem) {
@@ -1239,14 +1163,22 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
   uint32_t* sp = stack_lo;  // first free word
   const bool split_mode = heavy(P, top[2], top[0]);
   if (split_mode) A.splits++;
+  // register-resident DFS (one inline site): the whole task if its top has <= 32 candidates,
+  // else every pushed child with <= 32 candidates
+  const uint32_t* reg = nullptr;
+  uint32_t* reg_scratch = stack_lo;
   if constexpr (LPE == 0) {
-    if (split_mode && (P.debug & 2) && split_parallel(P, T, top, lmap, A, stack_lo, stack_hi)) return;
-    if (top[0] <= 32) {  // the whole task fits the register-resident DFS
-      run_reg(P, T, top, lmap, A, (RegLevel*)smem, stack_lo, stack_hi, split_mode, smem);
-      return;
-    }
+    if (top[0] <= 32) reg = top;
   }
   while (true) {
+    if constexpr (LPE == 0) {
+      if (reg) {
+        run_reg(P, T, reg, lmap, A, (RegLevel*)smem, reg_scratch, stack_hi, split_mode && reg == top, smem);
+        if (reg == top) return;
+        reg = nullptr;
+        continue;
+      }
+    }
     __syncwarp();
     const uint32_t i = cur[3];
     if (i >= cur[0]) {  // all candidates of this node traversed: pop (Alg 2 L4)
@@ -1274,7 +1206,8 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     }
     if constexpr (LPE == 0) {
       if (r == 2 && ch[0] <= 32) {  // the child's subtree fits the register-resident DFS
-        run_reg(P, T, ch, lmap, A, (RegLevel*)smem, align4(ch + rec_words(T, ch)), stack_hi, false, smem);
+        reg = ch;
+        reg_scratch = align4(ch + rec_words(T, ch));
         continue;
       }
     }
@@ -1290,7 +1223,7 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
   }
 }
 
-__device__ void dispatch_task(const Params& P, TaskCtx& T, uint32_t* top, uint32_t* lo, uint32_t* hi,
+__device__ GMBE_NI_IF(GMBE_NI_DISPATCH) void dispatch_task(const Params& P, TaskCtx& T, uint32_t* top, uint32_t* lo, uint32_t* hi,
                               uint32_t lmap, Acc& A, unsigned long long* smem) {
   if (T.W <= 2) {
     small_task_init(P, T, lmap);
@@ -1303,12 +1236,15 @@ __device__ void dispatch_task(const Params& P, TaskCtx& T, uint32_t* top, uint32
 }
 
 // ---------------------------------------------------------------- root task (a3)
-// Root v_s (rank r): L_r = N(v_s); wedge scan of N2(v_s) with k(v) = |N(v) ∩ L_r|.
-__device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
+// Root v_s (rank r): L_r = N(v_s); wedge scan of N2(v_s) with k(v) = |N(v) ∩ L_r|.  Emits the root
+// biclique and, if it has candidates, prepares its node record as a task (Tc, *top, stack from *lo)
+// for the caller's single dispatch site; returns whether it did.
+__device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A, TaskCtx& Tc,
+                                                  uint32_t** top, uint32_t** lo) {
   const uint32_t lane = lane_id();
   const DevGraph& g = P.g;
   const uint32_t lb = g.off_v[r], l = g.off_v[r + 1] - lb;
-  if (l == 0) return;  // isolated vertex: in no biclique (A17)
+  if (l == 0) return false;  // isolated vertex: in no biclique (A17)
   const uint32_t* Lr = g.adj_v + lb;
   uint32_t wp = 0;
   for (uint32_t j = lane; j < l; j += 32) {
@@ -1320,7 +1256,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
   const uint32_t T = next_pow2(max(64u, 2u * wedges));
   if (T > P.tmax || wedges > P.omax) {
     if (lane == 0) atomicOr(&P.ctrl->error, kErrArena);
-    return;
+    return false;
   }
   const uint32_t shift = 32 - (31 - __clz(T)), mask = T - 1;
   uint32_t* keys = M.keys;
@@ -1546,7 +1482,6 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
         rec[7] = (uint32_t)(sr >> 32);
       }
       __syncwarp();
-      TaskCtx Tc;
       Tc.map = Lr;
       Tc.W = W;
       Tc.W4 = W4;
@@ -1571,10 +1506,11 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
         }
       }
       PH_STOP(A, 3);
-      dispatch_task(P, Tc, rec, align4(rec + rec_need), M.dyn_end, l, A, M.sm_sort);
+      *top = rec;
+      *lo = align4(rec + rec_need);
     }
   }
-  // leave the table clean for the next root
+  // leave the table clean for the next root (the task no longer needs it)
   __syncwarp();
   for (uint32_t j = lane; j < nocc; j += 32) {
     const uint32_t s = M.occ[j];
@@ -1582,6 +1518,7 @@ __device__ void run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A) {
     vals[s] = 0;
   }
   __syncwarp();
+  return *top != nullptr;
 }
 
 __device__ __forceinline__ unsigned long long globaltimer() {
@@ -1594,7 +1531,7 @@ __device__ __forceinline__ uint32_t smid() {
   asm("mov.u32 %0, %%smid;" : "=r"(v));
   return v;
 }
-// profiling timeline: one record per root / task / descriptor (kind 0 / 1 / 2)
+// profiling timeline: one record per root / task (kind 0 / 1)
 // info = nodes generated by the record << 32 | min(|L_top|, 65535) << 16 | min(|C_top|, 65535)
 __device__ void timeline_rec(const Params& P, uint32_t kind, uint32_t root, unsigned long long t0,
                              unsigned long long info) {
@@ -1610,50 +1547,6 @@ __device__ void timeline_rec(const Params& P, uint32_t kind, uint32_t root, unsi
 }
 __device__ __forceinline__ unsigned long long tl_info(unsigned long long nodes, uint32_t l, uint32_t c) {
   return (nodes << 32) | ((unsigned long long)min(l, 65535u) << 16) | min(c, 65535u);
-}
-
-// Children G[a..b) of a published split node (see split_parallel), each followed by its subtree.
-__device__ void run_descriptor(const Params& P, const uint32_t* desc, WarpMem& M, Acc& A) {
-  const uint32_t lane = lane_id();
-  uint32_t* s = pool_ptr(P, desc[1]);
-  const uint32_t a = desc[2], b = desc[3];
-  TaskCtx Tc;
-  Tc.W = s[0];
-  const uint32_t lmap = s[1];
-  Tc.root = s[2];
-  const uint32_t rlen = s[3];
-  Tc.W4 = r4(Tc.W);
-  Tc.E = r4(Tc.W + 2);
-  Tc.map = s + kHdr;
-  Tc.rlist = M.rbuf;
-  Tc.auxref = s[5];
-  Tc.ncw = s[6];
-  Tc.cols = s[7] == 1 ? pool_ptr(P, Tc.auxref - 1) : nullptr;
-  Tc.gx = s[7] == 2 ? pool_ptr(P, Tc.auxref - 1) : nullptr;
-  small_task_init(P, Tc, lmap);
-  uint32_t* node = s + s[4];
-  const uint32_t n = node[0];
-  const uint32_t* dom = node + kHdr + 4 + 4 * n;
-  const uint32_t* G = dom + r4(n);
-  const long long c0 = clock64();
-  for (uint32_t t = a; t < b; t++) {
-    if (M.rbuf) {
-      for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
-      __syncwarp();
-    }
-    uint32_t* ch = M.dyn;
-    if (!fits(P, ch + kHdr + 4 + 4 * n + 4ull * 32 * Tc.W + 16, M.dyn_end)) return;
-    const int r = gen_child_small(P, Tc, node, G[t], ch, A, M.sm_sort, dom);
-    if (r == 2) {
-      if (lane == 0) {
-        ch[3] = 0;
-        ch[4] = kNone;
-      }
-      __syncwarp();
-      run_task<0>(P, Tc, ch, align4(ch + kHdr + 4 + 4 * ch[0]), M.dyn_end, lmap, A, M.sm_sort);
-    }
-  }
-  if (P.per_root_cycles && lane == 0) atomicAdd(P.per_root_cycles + Tc.root, (unsigned long long)(clock64() - c0));
 }
 
 #ifndef GMBE_MIN_BLOCKS
@@ -1676,7 +1569,14 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
   bool roots_done = false, is_hungry = false;
   uint32_t idle = 0;
   while (true) {
-    // 1. split subtasks first (Alg 4 L3-4)
+    // work item: a queued split subtask first (Alg 4 L3-4), else the next root (Alg 4 L6, heaviest =
+    // highest rank first); both end in the single dispatch site below
+    TaskCtx Tc;
+    uint32_t* top = nullptr;
+    uint32_t* lo = M.dyn;
+    uint32_t lmap = 0, kind = 2, item = 0, tl_l = 0, tl_c = 0;
+    const long long c0 = P.per_root_cycles ? clock64() : 0;
+    const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
     uint32_t task = kNone;
     if (lane == 0) task = queue_pop(P);
     task = __shfl_sync(GMBE_FULL, task, 0);
@@ -1688,17 +1588,8 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       PH_START(A);
       __threadfence();  // acquire: the task was written on another SM
       uint32_t* s = pool_ptr(P, task);
-      if (s[0] == kDescMagic) {
-        const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
-        run_descriptor(P, s, M, A);
-        if (P.timeline) timeline_rec(P, 2, 0, g0, tl_info(A.nodes - n0, 0, s[3] - s[2]));
-        if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
-        idle = 0;
-        continue;
-      }
-      TaskCtx Tc;
       Tc.W = s[0];
-      const uint32_t lmap = s[1];
+      lmap = s[1];
       Tc.root = s[2];
       const uint32_t rlen = s[3];
       Tc.W4 = r4(Tc.W);
@@ -1713,20 +1604,12 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
         for (uint32_t j = lane; j < rlen; j += 32) M.rbuf[j] = s[kHdr + r4(lmap) + j];
       __syncwarp();
       PH_STOP(A, 15);
-      const long long c0 = clock64();
-      const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
-      const uint32_t tl_l = s[s[4] + 2], tl_c = s[s[4]];
-      dispatch_task(P, Tc, s + s[4], M.dyn, M.dyn_end, lmap, A, M.sm_sort);
-      if (P.timeline) timeline_rec(P, 1, Tc.root, g0, tl_info(A.nodes - n0, tl_l, tl_c));
-      if (P.per_root_cycles && lane == 0)
-        atomicAdd(P.per_root_cycles + Tc.root, (unsigned long long)(clock64() - c0));
-      __syncwarp();
-      if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
-      idle = 0;
-      continue;
-    }
-    // 2. next root (Alg 4 L6), heaviest (highest rank) first
-    if (!roots_done) {
+      top = s + s[4];
+      kind = 1;
+      item = Tc.root;
+      tl_l = top[2];
+      tl_c = top[0];
+    } else if (!roots_done) {
       unsigned long long t = 0;
       if (lane == 0) {
         atomicAdd(&P.ctrl->pending.v, 1ull);
@@ -1735,21 +1618,26 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       t = __shfl_sync(GMBE_FULL, t, 0);
       if (t < P.n_roots) {
         const uint32_t rk = P.part_index + (P.n_roots - 1 - (uint32_t)t) * P.part_count;
-        const long long c0 = clock64();
-        const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
-        run_root(P, rk, M, A);
-        if (P.timeline)
-          timeline_rec(P, 0, rk, g0, tl_info(A.nodes - n0, P.g.off_v[rk + 1] - P.g.off_v[rk], 0));
-        if (P.per_root_cycles && lane == 0)
-          atomicAdd(P.per_root_cycles + rk, (unsigned long long)(clock64() - c0));
-        __syncwarp();
+        kind = 0;
+        item = rk;
+        if (run_root(P, rk, M, A, Tc, &top, &lo)) lmap = top[2];
+        tl_l = P.timeline ? P.g.off_v[rk + 1] - P.g.off_v[rk] : 0;
+      } else {
         if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
-        idle = 0;
-        continue;
+        roots_done = true;
       }
-      if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
-      roots_done = true;
     }
+    if (kind != 2) {
+      if (top) dispatch_task(P, Tc, top, lo, M.dyn_end, lmap, A, M.sm_sort);
+      if (P.timeline) timeline_rec(P, kind, item, g0, tl_info(A.nodes - n0, tl_l, tl_c));
+      if (P.per_root_cycles && lane == 0)
+        atomicAdd(P.per_root_cycles + item, (unsigned long long)(clock64() - c0));
+      __syncwarp();
+      if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
+      idle = 0;
+      continue;
+    }
+    if (!roots_done) continue;
     // 3. termination: all roots issued and nothing queued or running
     unsigned long long pend = 0;
     if (lane == 0) pend = ld_volatile(&P.ctrl->pending.v);

@@ -178,6 +178,26 @@ def test_split_and_schedule_invariance(gmbe, dense_case):
         g.free()
 
 
+def test_donation_invariance(gmbe, dense_case):
+    """Dynamic donation (debug bit 8: donate at every opportunity, bit 4: never) hands the remaining
+    children of a warp's shallowest level to the queue; the tree, the counters and the records must
+    be those of the canonical tree (DESIGN.md §5.2 "Dynamic donation")."""
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        for dbg in (8, 4, 12):
+            r = g.enumerate(debug=dbg, records=True)
+            _same(r, o)
+            assert r.algo_bytes_cand == o.algo_bytes_cand
+            assert r.bicliques == sorted(o.bicliques)
+            assert (r.donations > 0) == (dbg == 8), (dbg, r.donations)
+        r = g.enumerate(debug=8, bound_height=1, bound_size=1, records=True)
+        _same(r, o)
+        assert r.bicliques == sorted(o.bicliques)
+    finally:
+        g.free()
+
+
 def test_parts_are_additive(gmbe, dense_case):
     nu, nv, e, o = dense_case
     g = gmbe.load(nu, nv, e)
@@ -242,5 +262,36 @@ def test_full_config_vs_oracle_golden(gmbe, name):
         assert (r.nodes, r.nonmax, r.roots_run) == (gd["nodes"], gd["nonmax"], gd["roots_run"])
         if "algo_bytes_cand" in gd:
             assert r.algo_bytes_cand == gd["algo_bytes_cand"]
+    finally:
+        g.free()
+
+
+@pytest.mark.parametrize("name,n", [("gh_work", 8), ("dblp", 8), ("gh", 2)])
+def test_full_config_shards_vs_golden(gmbe, name, n):
+    """The bench's multi-GPU launch configuration (root shard i of n per rank, one all-reduce):
+    the shards' sums equal the whole-graph golden bit-exactly."""
+    gd = _gold_cfg()[name]
+    nu, nv, e = make_config(name)
+    g = gmbe.load(nu, nv, e)
+    try:
+        rs = [g.enumerate(part=(i, n)) for i in range(n)]
+        assert sum(r.count for r in rs) == gd["count"]
+        assert sum(r.checksum for r in rs) % (1 << 64) == int(gd["checksum"], 16)
+        assert sum(r.nodes for r in rs) == gd["nodes"]
+        assert sum(r.nonmax for r in rs) == gd["nonmax"]
+    finally:
+        g.free()
+
+
+@pytest.mark.parametrize("name", ["gh", "yg"])
+def test_full_config_forced_donation(gmbe, name):
+    gd = _gold_cfg()[name]
+    nu, nv, e = make_config(name)
+    g = gmbe.load(nu, nv, e)
+    try:
+        r = g.enumerate(debug=8)
+        assert r.donations > 0
+        assert (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16))
+        assert (r.nodes, r.nonmax, r.roots_run) == (gd["nodes"], gd["nonmax"], gd["roots_run"])
     finally:
         g.free()
