@@ -162,6 +162,9 @@ struct WarpMem {
   uint32_t* keys;               // clean hash table keys (EMPTY)
   unsigned long long* vals;     // clean hash table values (0)
   uint32_t* occ;                // occupied slots of the current root
+  uint32_t* skeys;              // the shared-memory table (kSmemTable slots)
+  unsigned long long* svals;
+  uint32_t* socc;
   uint32_t* dyn;                // dynamic region: root record, node stack, scratch
   uint32_t* dyn_end;
   uint32_t* rbuf;
@@ -205,6 +208,18 @@ __device__ __forceinline__ bool fits(const Params& P, const uint32_t* p, const u
 }
 
 // ---------------------------------------------------------------- per-warp hash table (a3)
+// Two instances per warp: a small one in shared memory (roots with <= kSmemTable/2 wedges, i.e.
+// almost every root of the light-tailed shapes) and the large one in the warp's HBM arena.  Both are
+// accessed through generic pointers: table reads are volatile (the slots are written by atomics, so
+// a global table must not be read through a stale L1 line), atomics resolve the address space.
+#ifndef GMBE_SMEM_TABLE
+#define GMBE_SMEM_TABLE 128
+#endif
+constexpr uint32_t kSmemTable = GMBE_SMEM_TABLE;
+__device__ __forceinline__ uint32_t ldv(const uint32_t* p) { return *(const volatile uint32_t*)p; }
+__device__ __forceinline__ unsigned long long ldv(const unsigned long long* p) {
+  return *(const volatile unsigned long long*)p;
+}
 __device__ __forceinline__ uint32_t ht_hash(uint32_t v, uint32_t shift) { return (v * 2654435761u) >> shift; }
 
 // warp-cooperative insert of v (lanes with act); new slots are appended to occ so the table can
@@ -216,7 +231,7 @@ __device__ __forceinline__ uint32_t ht_insert_warp(uint32_t* keys, uint32_t shif
   while (__any_sync(GMBE_FULL, pend)) {
     bool ins = false;
     if (pend) {
-      const uint32_t k = __ldcg(keys + h);
+      const uint32_t k = ldv(keys + h);
       if (k == v) {
         slot = h;
         pend = false;
@@ -242,7 +257,7 @@ __device__ __forceinline__ uint32_t ht_insert_warp(uint32_t* keys, uint32_t shif
 __device__ __forceinline__ uint32_t ht_find(const uint32_t* keys, uint32_t shift, uint32_t mask, uint32_t v) {
   uint32_t h = ht_hash(v, shift);
   while (true) {
-    const uint32_t k = __ldcg(keys + h);
+    const uint32_t k = ldv(keys + h);
     if (k == v) return h;
     if (k == GMBE_EMPTY) return kNone;
     h = (h + 1) & mask;
@@ -586,36 +601,6 @@ __device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_cols_is_r(const TaskCtx& T, cons
   return count == need;
 }
 
-// Alg 2 L14 with the root's Γ index gx (universe <= 64 bits, L' = lm): Γ(L') ⊆ {v_s} ∪ {x adjacent to
-// u*} for the lowest-degree u* ∈ L'; count the x whose row covers L'.  |Γ(L')| <= deg(u*), so
-// deg(u*) == |R'| proves maximality at once.
-__device__ bool gamma_gx_is_r(const uint32_t* gx, unsigned long long lm, uint32_t rlen) {
-  const uint32_t lane = lane_id();
-  const uint32_t nx = gx[0], l = gx[1];
-  const unsigned long long* xrow = (const unsigned long long*)(gx + 4);
-  const uint32_t* coff = gx + 4 + 2 * nx;
-  const uint32_t* cx = coff + r4(l + 1);
-  // j* = argmin over members of |list_j| (= deg(u_j) - 1)
-  uint32_t key = 0xffffffffu;
-  for (uint32_t j = lane; j < l; j += 32)
-    if ((lm >> j) & 1ull) key = min(key, ((coff[j + 1] - coff[j]) << 7) | j);
-  key = __reduce_min_sync(GMBE_FULL, key);
-  const uint32_t js = key & 127u, len = key >> 7;
-  if (len + 1 == rlen) return true;
-  uint32_t count = 1;  // v_s
-  const uint32_t* lst = cx + coff[js];
-  for (uint32_t b = 0; b < len; b += 32) {
-    bool full = false;
-    if (b + lane < len) {
-      const unsigned long long row = xrow[lst[b + lane]];
-      full = (row & lm) == lm;
-    }
-    count += __popc(__ballot_sync(GMBE_FULL, full));
-    if (count > rlen) return false;
-  }
-  return count == rlen;
-}
-
 // ---------------------------------------------------------------- child generation (a4, a5)
 // Generate the child of node `par` via its candidate i into `ch` (Alg 2 L6-16).  The parent's later
 // candidates are compacted in place (Thm 4.1 prunes removed), so par[0] shrinks.
@@ -718,10 +703,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
     while (!lpm[w]) w++;
     const uint32_t u = T.map[w * 32 + __ffs(lpm[w]) - 1];
     maximal = P.g.off_u[u + 1] - P.g.off_u[u] == rlen;
-  } else if (T.gx) {
-    const unsigned long long lm = W == 1 ? lpm[0] : ((unsigned long long)lpm[1] << 32) | lpm[0];
-    maximal = gamma_gx_is_r(T.gx, lm, rlen);
-  } else if (T.cols) {
+  } else if (T.cols) {  // (W > 2 here: the gx index only exists for universes <= 64 bits)
     maximal = gamma_cols_is_r(T, lpm, W, rlen);
   } else {
     maximal = gamma_is_r(P, lpm, W, T.map, lc, rlen, gscr, smem);
@@ -794,7 +776,10 @@ __device__ void small_task_init(const Params& P, TaskCtx& T, uint32_t lmap) {
   }
 }
 
-// maximality with gx and lane-resident list offsets (see gamma_gx_is_r)
+// Alg 2 L14 with the root's Γ index gx (universe <= 64 bits, L' = lm): Γ(L') ⊆ {v_s} ∪ X2 for
+// |L'| >= 2.  |X2| <= 64: count the lane-resident rows covering L'.  Otherwise walk the X2 list of the
+// member u* with the shortest list: |Γ(L')| <= 1 + |list(u*)|, so equality with |R'| proves
+// maximality at once; else count the listed rows covering L'.
 __device__ __forceinline__ bool gamma_gx_small(const TaskCtx& T, unsigned long long lm, uint32_t rlen) {
   const uint32_t lane = lane_id();
   if (T.nx <= 64) {  // lane-resident X2 rows: |Γ(L')| = 1 + #rows covering L'
@@ -1259,15 +1244,17 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
     return false;
   }
   const uint32_t shift = 32 - (31 - __clz(T)), mask = T - 1;
-  uint32_t* keys = M.keys;
-  unsigned long long* vals = M.vals;
+  const bool stab = kSmemTable && T <= kSmemTable;  // shared-memory table
+  uint32_t* keys = stab ? M.skeys : M.keys;
+  unsigned long long* vals = stab ? M.svals : M.vals;
+  uint32_t* occl = stab ? M.socc : M.occ;
   const bool small = l <= 64;  // rows (<= 64 bits) straight from the table
   PH_START(A);
   // pass 1 (Alg 3 L2-3)
   uint32_t nocc = 0;
   for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
     const bool a = act && v != r;
-    const uint32_t h = ht_insert_warp(keys, shift, mask, v, a, M.occ, nocc);
+    const uint32_t h = ht_insert_warp(keys, shift, mask, v, a, occl, nocc);
     if (a) {
       if (small) atomicOr(vals + h, 1ull << i);
       else atomicAdd(vals + h, 1ull);
@@ -1286,11 +1273,11 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   for (uint32_t b = 0; b < nocc && sort_fits; b += 32) {
     const uint32_t j = b + lane;
     const bool occ = j < nocc;
-    const uint32_t s = occ ? M.occ[j] : 0;
-    const uint32_t v = occ ? __ldcg(keys + s) : 0;
+    const uint32_t s = occ ? occl[j] : 0;
+    const uint32_t v = occ ? ldv(keys + s) : 0;
     uint32_t c = 0;
     if (occ) {
-      const unsigned long long x = __ldcg(vals + s);
+      const unsigned long long x = ldv(vals + s);
       c = small ? __popcll(x) : (uint32_t)x;
     }
     const bool isR = occ && c == l;
@@ -1349,16 +1336,17 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
       uint32_t n2 = 0;
       for (uint32_t b = 0; b < nocc; b += 32) {
         const uint32_t x = b + lane;
-        const unsigned long long row = x < nocc ? __ldcg(vals + M.occ[x]) : 0ull;
+        const unsigned long long row = x < nocc ? ldv(vals + occl[x]) : 0ull;
         const bool is2 = __popcll(row) >= 2;
         const uint32_t bal = __ballot_sync(GMBE_FULL, is2);
         if (is2) xrow[n2 + __popc(bal & lanemask_lt())] = row;
         n2 += __popc(bal);
       }
       __syncwarp();
-      // list lengths: lane j counts universe vertex j (cnt0) and j + 32 (cnt1)
+      // list lengths: lane j counts universe vertex j (cnt0) and j + 32 (cnt1).  With |X2| <= 64 the
+      // rows are lane-resident in every task of this root (small_task_init) and no list is needed.
       uint32_t cnt0 = 0, cnt1 = 0;
-      for (uint32_t b = 0; b < nx2; b += 32) {
+      for (uint32_t b = 0; b < nx2 && nx2 > 64; b += 32) {
         const unsigned long long row = b + lane < nx2 ? xrow[b + lane] : 0ull;
         unsigned long long any = ((unsigned long long)__reduce_or_sync(GMBE_FULL, (uint32_t)(row >> 32)) << 32) |
                                  __reduce_or_sync(GMBE_FULL, (uint32_t)row);
@@ -1389,7 +1377,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
       }
       if (lane == 0 && l == 64) coff[64] = carry;
       __syncwarp();
-      for (uint32_t b = 0; b < nx2; b += 32) {
+      for (uint32_t b = 0; b < nx2 && nx2 > 64; b += 32) {
         const uint32_t x = b + lane;
         const unsigned long long row = x < nx2 ? xrow[x] : 0ull;
         unsigned long long any = ((unsigned long long)__reduce_or_sync(GMBE_FULL, (uint32_t)(row >> 32)) << 32) |
@@ -1420,7 +1408,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
       for (uint32_t j = lane; j < nC; j += 32) {
         const unsigned long long kv = sortbuf[j];
         const uint32_t s = (uint32_t)kv;
-        const unsigned long long x = __ldcg(vals + s);
+        const unsigned long long x = ldv(vals + s);
         uint32_t* ee = ent + (size_t)j * E;
         if (small) {
           ee[0] = (uint32_t)x;
@@ -1441,8 +1429,8 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
         uint32_t n2 = 0;
         for (uint32_t b = 0; b < nocc; b += 32) {
           const uint32_t x = b + lane;
-          const uint32_t s2 = x < nocc ? M.occ[x] : 0u;
-          const unsigned long long v2 = x < nocc ? __ldcg(vals + s2) : 0ull;
+          const uint32_t s2 = x < nocc ? occl[x] : 0u;
+          const unsigned long long v2 = x < nocc ? ldv(vals + s2) : 0ull;
           const bool isc = (v2 & kCTag) != 0;
           const uint32_t k = isc ? ent[(size_t)(uint32_t)(v2 & 0x7fffffffull) * E + W + 1] : (uint32_t)v2;
           const bool is2 = x < nocc && k >= 2;
@@ -1457,7 +1445,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
         for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
           if (act && v != r) {
             const uint32_t h = ht_find(keys, shift, mask, v);
-            const unsigned long long x = __ldcg(vals + h);
+            const unsigned long long x = ldv(vals + h);
             const uint32_t xi = (uint32_t)(x >> 32);
             if (want_cols && xi) atomicOr(cols + (size_t)i * ncw + ((xi - 1) >> 5), 1u << ((xi - 1) & 31));
             if (x & 0x80000000ull) atomicOr(ent + (size_t)(x & 0x7fffffffull) * E + (i >> 5), 1u << (i & 31));
@@ -1513,7 +1501,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   // leave the table clean for the next root (the task no longer needs it)
   __syncwarp();
   for (uint32_t j = lane; j < nocc; j += 32) {
-    const uint32_t s = M.occ[j];
+    const uint32_t s = occl[j];
     keys[s] = GMBE_EMPTY;
     vals[s] = 0;
   }
@@ -1554,6 +1542,9 @@ __device__ __forceinline__ unsigned long long tl_info(unsigned long long nodes, 
 #endif
 __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
   __shared__ unsigned long long s_sort[8][kSmemSort];
+  __shared__ unsigned long long s_tvals[8][kSmemTable ? kSmemTable : 1];
+  __shared__ uint32_t s_tkeys[8][kSmemTable ? kSmemTable : 1];
+  __shared__ uint32_t s_tocc[8][kSmemTable ? kSmemTable / 2 : 1];
   const uint32_t lane = lane_id();
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   uint32_t* base = P.arena + (uint64_t)gw * P.arena_words;
@@ -1565,6 +1556,14 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
   M.dyn_end = base + P.arena_words;
   M.rbuf = P.rbuf ? P.rbuf + (uint64_t)gw * P.rbuf_words : nullptr;
   M.sm_sort = s_sort[threadIdx.x >> 5];
+  M.skeys = s_tkeys[threadIdx.x >> 5];
+  M.svals = s_tvals[threadIdx.x >> 5];
+  M.socc = s_tocc[threadIdx.x >> 5];
+  for (uint32_t j = lane; j < kSmemTable; j += 32) {
+    M.skeys[j] = GMBE_EMPTY;
+    M.svals[j] = 0;
+  }
+  __syncwarp();
   Acc A = {};
   bool roots_done = false, is_hungry = false;
   uint32_t idle = 0;
