@@ -78,8 +78,10 @@ struct Params {
   unsigned long long* per_root;
   unsigned long long* per_root_cycles;
   uint32_t profile;
-  uint32_t debug;  // opts.reserved0 bits (tests / experiments): 4 = no donation, 8 = donate whenever possible
+  uint32_t debug;  // opts.reserved0 bits (tests / experiments): 4 = no donation, 8 = donate whenever possible,
+                   // 16 = no thread-level tier (run_thr), 32 = path statistics into ctrl.phase
   uint32_t donate;  // dynamic donation to idle warps (donate_reg)
+  uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.reserved1 overrides; experiments)
   unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1, info]*
   uint64_t timeline_cap;
 };
@@ -120,7 +122,8 @@ struct TaskCtx {
   uint32_t* rlist;      // R-list stack (output only)
   // Γ index of the root (maximality count without binary searches), one of:
   //   gx  (universe <= 64 bits): [nx, l, -, -] | xrow u64[nx] (row of each X2 vertex x over the
-  //        universe) | coff u32[l+1] | cx u32[] (X2 indices adjacent to universe vertex j)
+  //        universe) | xid u32[r4(nx)] (rank of x) | coff u32[l+1] | cx u32[] (X2 indices adjacent
+  //        to universe vertex j)
   //   cols (larger universes): cols[j*ncw ..] = bitmap of the X2 vertices adjacent to vertex j
   // X2 = the root's 2-hop vertices adjacent to >= 2 universe vertices (the only ones that can cover
   // an L' with |L'| >= 2).
@@ -132,6 +135,7 @@ struct TaskCtx {
   // lane-resident copies for universes <= 64 bits (universe vertices lane and lane + 32), filled by
   // small_task_init: Γ-list offsets / lengths and the checksum hashes of the universe vertices
   uint32_t go0, go1, gl0, gl1;
+  uint32_t dg0, dg1;          // degrees of the universe vertices (run_thr's |L'| = 1 test)
   unsigned long long hu0, hu1;
   uint32_t nx;                // gx: |X2|; <= 64: the X2 rows are lane-resident in xr0 / xr1
   unsigned long long xr0, xr1;
@@ -752,6 +756,15 @@ __device__ void small_task_init(const Params& P, TaskCtx& T, uint32_t lmap) {
   T.go0 = T.go1 = T.gl0 = T.gl1 = 0;
   T.hu0 = lane < lmap ? gmbe_hid(T.map[lane], P.hu_side) : 0ull;
   T.hu1 = lane + 32 < lmap ? gmbe_hid(T.map[lane + 32], P.hu_side) : 0ull;
+  T.dg0 = T.dg1 = 0;
+  if (lane < lmap) {
+    const uint32_t u = T.map[lane];
+    T.dg0 = P.g.off_u[u + 1] - P.g.off_u[u];
+  }
+  if (lane + 32 < lmap) {
+    const uint32_t u = T.map[lane + 32];
+    T.dg1 = P.g.off_u[u + 1] - P.g.off_u[u];
+  }
   T.gxl = nullptr;
   T.nx = kNone;
   T.xr0 = T.xr1 = 0;
@@ -762,7 +775,7 @@ __device__ void small_task_init(const Params& P, TaskCtx& T, uint32_t lmap) {
       if (lane < T.nx) T.xr0 = xrow[lane];
       if (lane + 32 < T.nx) T.xr1 = xrow[lane + 32];
     }
-    const uint32_t* coff = T.gx + 4 + 2 * T.gx[0];
+    const uint32_t* coff = T.gx + 4 + 2 * T.gx[0] + r4(T.gx[0]);
     const uint32_t l = T.gx[1];
     T.gxl = coff + r4(l + 1);
     if (lane < l) {
@@ -1140,9 +1153,398 @@ __device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& 
   }
 }
 
+// ---------------------------------------------------------------- thread-level subtrees
+// The same nodes as run_reg (<= 32 candidates over a <= 64-bit universe), walked one subtree per
+// THREAD instead of one node per warp: a node is generated by one lane with scalar AND/POPC over
+// the job's candidate rows in shared memory, so the 32 lanes of a warp generate up to 32 nodes at a
+// time (Alg 2 unchanged; the paper's warp-per-procedure granularity, is kept for the
+// heavier node layouts).  Work is spread inside the warp by donation: an idle lane receives the
+// remaining children of a busy lane's shallowest stacked level (the node (L_k, R_k, remaining
+// candidates of level k) -- its children, later sets and Thm 4.1 marks are exactly the ones the
+// donor would have generated, so the tree and every counter stay those of the canonical tree).
+// Maximality (Alg 2 L14), |L'| >= 2: L' is non-maximal iff some x ∈ Γ(L') lies outside R'.  Under
+// the job (L0, R_job = Γ(L0), candidates C0) such an x is either a job candidate outside R' (tested
+// with per-vertex candidate columns) or one of the job's Q patterns N(x) ∩ L0 (x ∈ X2 \ (R_job ∪ C0),
+// deduplicated, reduced to the maximal ones above 64; tested with per-vertex pattern columns):
+// both are one AND per member of L'.  |L'| = 1: deg(u) == |R'|.
+struct ThrSmem {
+  unsigned long long row[32];  // candidate rows over the universe (the job's top node)
+  unsigned long long hv[32];   // hV of each candidate
+  unsigned long long hu[64];   // hU of each universe vertex
+  uint32_t deg[64];            // degree of each universe vertex
+  uint32_t id[32];             // rank of each candidate
+};
+struct ThrLevel {
+  unsigned long long L, SR;
+  uint32_t C, Rm, next, pad;
+};
+
+// one output record from one lane: L' = bits of lp over map, R' = the job's R list + candidates rm
+__device__ void write_record_thr(const Params& P, const TaskCtx& T, const ThrSmem* ts, unsigned long long lp,
+                                 uint32_t nl, uint32_t rlen0, uint32_t rm, uint32_t nr) {
+  const unsigned long long need = 2ull + nl + nr;
+  const unsigned long long rec = atomicAdd(&P.ctrl->out_rec, 1ull);
+  const unsigned long long off = atomicAdd(&P.ctrl->out_ids, need);
+  if (rec >= P.out_offsets_cap || off + need > P.out_ids_cap) {
+    atomicOr(&P.ctrl->truncated, 1u);
+    if (rec < P.out_offsets_cap) P.out_offsets[rec] = ~0ull;
+    return;
+  }
+  uint32_t* o = P.out_ids + off;
+  const bool sw = P.hu_side != 0;
+  uint32_t* lpos = sw ? o + 2 + nr : o + 2;
+  uint32_t* rpos = sw ? o + 2 : o + 2 + nl;
+  o[0] = sw ? nr : nl;
+  o[1] = sw ? nl : nr;
+  uint32_t t = 0;
+  for (; t < rlen0; t++) rpos[t] = P.g.rank2id[T.rlist[t]];
+  for (uint32_t m = rm; m; m &= m - 1) rpos[t++] = P.g.rank2id[ts->id[__ffs(m) - 1]];
+  t = 0;
+  for (unsigned long long m = lp; m; m &= m - 1) lpos[t++] = T.map[__ffsll(m) - 1];
+  P.out_offsets[rec] = off;
+}
+
+// Publish lane `src`'s stacked level k (its remaining children) as a subtask for idle warps
+// (cross-warp donation, see donate_reg).  Warp-cooperative; returns whether it was published.
+__device__ bool donate_thr(const Params& P, const TaskCtx& T, uint32_t lmap, Acc& A, const ThrSmem* ts,
+                           uint32_t nC, uint32_t rlen0, uint32_t src, unsigned long long Lk, unsigned long long SRk,
+                           uint32_t Ck, uint32_t Rmk, uint32_t nextk, uint32_t* scratch, const uint32_t* scratch_end) {
+  const uint32_t lane = lane_id();
+  const bool w2 = T.W == 2;
+  Lk = shfl64(Lk, src);
+  SRk = shfl64(SRk, src);
+  Ck = __shfl_sync(GMBE_FULL, Ck, src);
+  Rmk = __shfl_sync(GMBE_FULL, Rmk, src);
+  nextk = __shfl_sync(GMBE_FULL, nextk, src);
+  const uint32_t av = Ck & (GMBE_FULL << nextk);
+  const uint32_t n = __popc(av);
+  const uint32_t words = kHdr + 4 + 4 * n;
+  if (scratch + words > scratch_end) return false;
+  uint4* ce = (uint4*)(scratch + kHdr + 4);
+  if (lane < nC && ((av >> lane) & 1u)) {
+    const unsigned long long xr = ts->row[lane] & Lk;
+    const uint32_t id = ts->id[lane], kc = __popcll(xr);
+    ce[__popc(av & lanemask_lt())] = w2 ? make_uint4((uint32_t)xr, (uint32_t)(xr >> 32), id, kc)
+                                        : make_uint4((uint32_t)xr, id, kc, 0);
+  }
+  const uint32_t rk = rlen0 + __popc(Rmk);
+  if (T.rlist && lane < nC && ((Rmk >> lane) & 1u)) T.rlist[rlen0 + __popc(Rmk & lanemask_lt())] = ts->id[lane];
+  if (lane == 0) {
+    scratch[0] = n;
+    scratch[1] = 0;
+    scratch[2] = __popcll(Lk);
+    scratch[3] = 0;
+    scratch[4] = kNone;
+    scratch[5] = rk;
+    scratch[6] = (uint32_t)SRk;
+    scratch[7] = (uint32_t)(SRk >> 32);
+    scratch[kHdr] = (uint32_t)Lk;
+    scratch[kHdr + 1] = (uint32_t)(Lk >> 32);
+    scratch[kHdr + 2] = 0;
+    scratch[kHdr + 3] = 0;
+  }
+  __syncwarp();
+  if (!task_publish(P, T, lmap, T.rlist ? rk : 0, scratch, words, A)) return false;
+  A.donations++;
+  return true;
+}
+
+#ifndef GMBE_NI_THR
+#define GMBE_NI_THR 0
+#endif
+#ifndef GMBE_THR_MIN_EST
+#define GMBE_THR_MIN_EST 16  // jobs with fewer adjacency bits (Σ(k-1)) stay on run_reg (setup > work)
+#endif
+// smem layout of the column store (the warp's s_sort slice, kSmemSort u64): [0, 128) pattern hash
+// table during setup, then [128, 256) = one ThrCol per universe vertex j
+struct ThrCol {
+  unsigned long long q;  // bit t: Q-pattern t contains j
+  uint32_t c, pad;       // bit c: job candidate c is adjacent to j
+};
+constexpr uint32_t kThrHash = 128;
+static_assert(kSmemSort * 8 >= kThrHash * 8 + 64 * sizeof(ThrCol), "column store exceeds the s_sort slice");
+__device__ __forceinline__ bool sorted_has(const uint32_t* a, uint32_t n, uint32_t x) {
+  uint32_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (a[mid] < x) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo < n && a[lo] == x;
+}
+// Returns false (nothing done) when the job does not fit this tier (no Γ index, too few candidates,
+// more than 64 Q patterns after reduction); the caller then runs it with run_reg.
+__device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& T, const uint32_t* rec, uint32_t lmap,
+                                                Acc& A, ThrSmem* ts, unsigned long long* smem, uint32_t* scratch,
+                                                const uint32_t* scratch_end) {
+  const uint32_t lane = lane_id();
+  const uint32_t nC = rec[0];
+  if (!T.gx) return false;
+  const bool w2 = T.W == 2;
+  uint4 x = make_uint4(0, 0, 0, 0);
+  if (lane < nC) x = ((const uint4*)(rec + kHdr + 4))[lane];
+  // job weight: adjacency bits beyond one per candidate (a candidate with k = 1 only yields a leaf)
+  if (warp_sum(lane < nC ? (w2 ? x.w : x.z) - 1u : 0u) < P.thr_min_est) return false;
+  const unsigned long long L0 = ((unsigned long long)rec[kHdr + 1] << 32) | rec[kHdr];
+  PH_START(A);
+  // the job's candidates (rank order) and universe
+  unsigned long long crow = 0;
+  if (lane < nC) {
+    crow = w2 ? (((unsigned long long)x.y << 32) | x.x) : x.x;
+    const uint32_t id = w2 ? x.z : x.y;
+    ts->row[lane] = crow;
+    ts->id[lane] = id;
+    ts->hv[lane] = P.g.hv[id];
+  }
+  ts->hu[lane] = T.hu0;
+  ts->hu[lane + 32] = T.hu1;
+  ts->deg[lane] = T.dg0;
+  ts->deg[lane + 32] = T.dg1;
+  unsigned long long* ht = smem;
+  for (uint32_t t = lane; t < kThrHash; t += 32) ht[t] = 0ull;
+  __syncwarp();
+  // Q patterns of the job: N(x) ∩ L0 for x ∈ X2 with |N(x) ∩ L0| >= 2 that is neither in R_job
+  // (N(x) ⊇ L0: the job node is maximal, so Γ(L0) = R_job) nor a job candidate; deduplicated.
+  // Under the job every such x lies outside R', and L' is non-maximal if one of them covers it.
+  const uint32_t nx = T.gx[0];
+  const unsigned long long* xrow = (const unsigned long long*)(T.gx + 4);
+  const uint32_t* xid = T.gx + 4 + 2 * nx;
+  bool over = false;
+  for (uint32_t b = 0; b < nx; b += 32) {
+    const uint32_t x = b + lane;
+    const unsigned long long p = x < nx ? xrow[x] & L0 : 0ull;
+    bool q = __popcll(p) >= 2 && p != L0;
+    if (q) q = !sorted_has(ts->id, nC, xid[x]);
+    if (q) {  // insert p (linear probing; 0 = empty)
+      uint32_t h = (uint32_t)((p * 0x9E3779B97F4A7C15ull) >> 57), n = 0;
+      while (true) {
+        const unsigned long long old = atomicCAS(ht + h, 0ull, p);
+        if (old == 0ull || old == p) break;
+        h = (h + 1) & (kThrHash - 1);
+        if (++n == kThrHash) {
+          over = true;
+          break;
+        }
+      }
+    }
+  }
+  __syncwarp();
+  if (__any_sync(GMBE_FULL, over)) return false;
+  // distinct patterns: compact the table to ht[0, npat); above 64, keep only the maximal ones (a
+  // pattern inside another covers no L' the other does not)
+  unsigned long long pk[4];
+  uint32_t npat = 0;
+#pragma unroll
+  for (int k = 0; k < 4; k++) {
+    pk[k] = ht[k * 32 + lane];
+    npat += __popc(__ballot_sync(GMBE_FULL, pk[k] != 0ull));
+  }
+  if (npat > 64) {
+    for (uint32_t t = 0; t < kThrHash; t++) {
+      const unsigned long long o = ht[t];  // broadcast read
+      if (!o) continue;
+#pragma unroll
+      for (int k = 0; k < 4; k++)
+        if ((pk[k] & o) == pk[k] && pk[k] != o) pk[k] = 0ull;
+    }
+  }
+  __syncwarp();
+  npat = 0;
+#pragma unroll
+  for (int k = 0; k < 4; k++) {
+    const uint32_t bal = __ballot_sync(GMBE_FULL, pk[k] != 0ull);
+    if (pk[k]) ht[npat + __popc(bal & lanemask_lt())] = pk[k];
+    npat += __popc(bal);
+  }
+  if (npat > 64) return false;
+  __syncwarp();
+  const unsigned long long q0 = lane < npat ? ht[lane] : 0ull, q1 = lane + 32 < npat ? ht[lane + 32] : 0ull;
+  __syncwarp();
+  ThrCol* cols = (ThrCol*)(smem + kThrHash);
+  for (unsigned long long m = L0; m; m &= m - 1) {
+    const uint32_t j = __ffsll(m) - 1;
+    const unsigned long long qj = __ballot_sync(GMBE_FULL, (q0 >> j) & 1ull) |
+                                  ((unsigned long long)__ballot_sync(GMBE_FULL, (q1 >> j) & 1ull) << 32);
+    const uint32_t cj = __ballot_sync(GMBE_FULL, (crow >> j) & 1ull);
+    if (lane == (j & 31)) {
+      cols[j].q = qj;
+      cols[j].c = cj;
+    }
+  }
+  __syncwarp();
+  PH_STOP(A, 13);
+  const uint32_t rlen0 = rec[5];
+  ThrLevel stk[32];
+  bool has = lane == 0;
+  unsigned long long L = L0, SR = ((unsigned long long)rec[7] << 32) | rec[6];
+  const uint32_t cand_all = nC >= 32 ? GMBE_FULL : ((1u << nC) - 1u);
+  uint32_t C = cand_all, next = 0, Rm = 0, d = 0, dmask = 0;
+  uint32_t n_nodes = 0, n_nonmax = 0, n_count = 0;
+  unsigned long long abytes = 0, cks = 0;
+#if GMBE_DONATE
+  uint32_t tick = 0;
+#endif
+  while (true) {
+    if (has) {  // pop (Alg 2 L4) until a node with an untraversed candidate
+      while (true) {
+        if (next < 32 && (C & (GMBE_FULL << next))) break;
+        if (d == 0) {
+          has = false;
+          break;
+        }
+        d--;
+        L = stk[d].L;
+        SR = stk[d].SR;
+        C = stk[d].C;
+        Rm = stk[d].Rm;
+        next = stk[d].next;
+        dmask &= ~(1u << d);
+      }
+    }
+    const uint32_t idle = __ballot_sync(GMBE_FULL, !has);
+    if (idle == GMBE_FULL) break;
+    if (idle) {  // in-warp donation: the r-th idle lane takes the shallowest level of the r-th donor
+      const uint32_t donors = __ballot_sync(GMBE_FULL, dmask != 0);
+      if (donors) {
+        const uint32_t nd = min(__popc(idle), __popc(donors));
+        unsigned long long gL = 0, gSR = 0;
+        uint32_t gC = 0, gRm = 0, gnext = 0;
+        if (dmask && __popc(donors & lanemask_lt()) < nd) {
+          const uint32_t k = __ffs(dmask) - 1;
+          gL = stk[k].L;
+          gSR = stk[k].SR;
+          gC = stk[k].C;
+          gRm = stk[k].Rm;
+          gnext = stk[k].next;
+          stk[k].next = 32;  // the remaining children of level k are no longer this lane's
+          dmask &= ~(1u << k);
+        }
+        const uint32_t ir = __popc(idle & lanemask_lt());
+        const bool take = !has && ir < nd;
+        const uint32_t src = take ? __fns(donors, 0, ir + 1) : lane;
+        gL = shfl64(gL, src);
+        gSR = shfl64(gSR, src);
+        gC = __shfl_sync(GMBE_FULL, gC, src);
+        gRm = __shfl_sync(GMBE_FULL, gRm, src);
+        gnext = __shfl_sync(GMBE_FULL, gnext, src);
+        if (take) {
+          has = true;
+          L = gL;
+          SR = gSR;
+          C = gC;
+          Rm = gRm;
+          next = gnext;
+          d = 0;
+          dmask = 0;
+        }
+      }
+    }
+#if GMBE_DONATE
+    if ((!idle || (P.debug & 8)) && P.donate && (++tick & 7) == 0 && hungry(P)) {  // cross-warp donation to idle warps
+      const uint32_t donors = __ballot_sync(GMBE_FULL, dmask != 0);
+      if (donors) {
+        const uint32_t src = __ffs(donors) - 1;
+        const uint32_t k = lane == src ? __ffs(dmask) - 1 : 0;
+        unsigned long long kL = 0, kSR = 0;
+        uint32_t kC = 0, kRm = 0, knext = 0;
+        if (lane == src) {
+          kL = stk[k].L;
+          kSR = stk[k].SR;
+          kC = stk[k].C;
+          kRm = stk[k].Rm;
+          knext = stk[k].next;
+        }
+        if (donate_thr(P, T, lmap, A, ts, nC, rlen0, src, kL, kSR, kC, kRm, knext, scratch, scratch_end) &&
+            lane == src) {
+          stk[k].next = 32;
+          dmask &= ~(1u << k);
+        }
+      }
+    }
+#endif
+    if (!has) continue;
+    // generate the child via the next candidate i (Alg 2 L6-13)
+    const uint32_t i = __ffs(C & (GMBE_FULL << next)) - 1;
+    next = i + 1;
+    const unsigned long long lp = L & ts->row[i];  // L' = L ∩ N(v')
+    const uint32_t lc = __popcll(lp);
+    const uint32_t later = i >= 31 ? 0u : (C & (GMBE_FULL << (i + 1)));
+    uint32_t pr = 0, ab = 0, cd = 0, ksum = 0;
+    unsigned long long srab = 0;
+    for (uint32_t m = later; m; m &= m - 1) {
+      const uint32_t c = __ffs(m) - 1;
+      const unsigned long long rc = ts->row[c];
+      const uint32_t kp = __popcll(rc & L), kc = __popcll(rc & lp);
+      const uint32_t bit = 1u << c;
+      ksum += kp;
+      if (kc == kp) pr |= bit;  // Thm 4.1
+      if (kc == lc) {           // absorbed into R'
+        ab |= bit;
+        srab += ts->hv[c];
+      } else if (kc) {
+        cd |= bit;
+      }
+    }
+    if (P.prune) C &= ~pr;
+    n_nodes++;
+    abytes += lc + ksum;
+    const uint32_t rl = rlen0 + __popc(Rm) + 1 + __popc(ab);
+    // maximality (Alg 2 L14): |Γ(L')| == |R'|
+    bool maximal;
+    if (lc == 1) {
+      maximal = ts->deg[__ffsll(lp) - 1] == rl;
+    } else {  // |L'| >= 2: no Q pattern and no job candidate outside R' may cover L'
+      const uint32_t outside = cand_all & ~(Rm | (1u << i) | ab);
+      unsigned long long qa = ~0ull;
+      uint32_t ca = GMBE_FULL;
+      for (unsigned long long m = lp; m; m &= m - 1) {
+        const ThrCol tc = cols[__ffsll(m) - 1];
+        qa &= tc.q;
+        ca &= tc.c;
+        if (!qa && !(ca & outside)) break;
+      }
+      maximal = !qa && !(ca & outside);
+    }
+    if (!maximal) {
+      n_nonmax++;
+      continue;
+    }
+    // Output(L', R') (Alg 2 L15)
+    unsigned long long sl = 0;
+    for (unsigned long long m = lp; m; m &= m - 1) sl += ts->hu[__ffsll(m) - 1];
+    const unsigned long long srn = SR + ts->hv[i] + srab;
+    const uint32_t rmn = Rm | (1u << i) | ab;
+    n_count++;
+    cks += pair_hash(P, sl, srn);
+    if (P.per_root) atomicAdd(P.per_root + T.root, 1ull);
+    if (T.rlist && P.out_ids) write_record_thr(P, T, ts, lp, lc, rlen0, rmn, rl);
+    if (!cd) continue;
+    // push (Alg 2 L16)
+    stk[d].L = L;
+    stk[d].SR = SR;
+    stk[d].C = C;
+    stk[d].Rm = Rm;
+    stk[d].next = next;
+    if (next < 32 && (C & (GMBE_FULL << next))) dmask |= 1u << d;
+    d++;
+    L = lp;
+    SR = srn;
+    C = cd;
+    Rm = rmn;
+    next = 0;
+  }
+  A.nodes += warp_sum(n_nodes);
+  A.nonmax += warp_sum(n_nonmax);
+  A.count += warp_sum(n_count);
+  A.abytes += 4ull * warp_sum64r(abytes);
+  A.checksum += warp_sum64r(cks);
+  PH_STOP(A, 4);
+  return true;
+}
+
 template <int LPE>
 __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint32_t* stack_lo, uint32_t* stack_hi,
-                         uint32_t lmap, Acc& A, unsigned long long* smem) {
+                         uint32_t lmap, Acc& A, unsigned long long* smem, ThrSmem* ts) {
   const uint32_t lane = lane_id();
   uint32_t* cur = top;
   uint32_t* sp = stack_lo;  // first free word
@@ -1158,7 +1560,18 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
   while (true) {
     if constexpr (LPE == 0) {
       if (reg) {
-        run_reg(P, T, reg, lmap, A, (RegLevel*)smem, reg_scratch, stack_hi, split_mode && reg == top, smem);
+        const bool st = split_mode && reg == top;  // heavy top: publish its children (run_reg)
+#ifndef GMBE_PROFILE
+        const unsigned long long n0 = A.nodes;
+#endif
+        const bool thr = !st && !(P.debug & 16) && run_thr(P, T, reg, lmap, A, ts, smem, reg_scratch, stack_hi);
+        if (!thr) run_reg(P, T, reg, lmap, A, (RegLevel*)smem, reg_scratch, stack_hi, st, smem);
+#ifndef GMBE_PROFILE
+        if ((P.debug & 32) && lane == 0) {  // path statistics (experiments): jobs / nodes per tier
+          atomicAdd(&P.ctrl->phase[thr ? 0 : 2], 1ull);
+          atomicAdd(&P.ctrl->phase[thr ? 1 : 3], A.nodes - n0);
+        }
+#endif
         if (reg == top) return;
         reg = nullptr;
         continue;
@@ -1209,15 +1622,15 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
 }
 
 __device__ GMBE_NI_IF(GMBE_NI_DISPATCH) void dispatch_task(const Params& P, TaskCtx& T, uint32_t* top, uint32_t* lo, uint32_t* hi,
-                              uint32_t lmap, Acc& A, unsigned long long* smem) {
+                              uint32_t lmap, Acc& A, unsigned long long* smem, ThrSmem* ts) {
   if (T.W <= 2) {
     small_task_init(P, T, lmap);
-    run_task<0>(P, T, top, lo, hi, lmap, A, smem);
+    run_task<0>(P, T, top, lo, hi, lmap, A, smem, ts);
   }
-  else if (T.W <= 4) run_task<4>(P, T, top, lo, hi, lmap, A, smem);  // W > 2 from here
-  else if (T.W <= 8) run_task<8>(P, T, top, lo, hi, lmap, A, smem);
-  else if (T.W <= 16) run_task<16>(P, T, top, lo, hi, lmap, A, smem);
-  else run_task<32>(P, T, top, lo, hi, lmap, A, smem);
+  else if (T.W <= 4) run_task<4>(P, T, top, lo, hi, lmap, A, smem, ts);  // W > 2 from here
+  else if (T.W <= 8) run_task<8>(P, T, top, lo, hi, lmap, A, smem, ts);
+  else if (T.W <= 16) run_task<16>(P, T, top, lo, hi, lmap, A, smem, ts);
+  else run_task<32>(P, T, top, lo, hi, lmap, A, smem, ts);
 }
 
 // ---------------------------------------------------------------- root task (a3)
@@ -1302,7 +1715,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   // universes <= 64 bits, columns otherwise (see TaskCtx).  x2 = position of x among X2 in occ order.
   const uint32_t ncw = (nx2 + 31) / 32;
   uint32_t* aux = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
-  const uint64_t aux_words = small ? 4ull + 2ull * nx2 + r4(l + 1) + sum2 : (uint64_t)l * ncw;
+  const uint64_t aux_words = small ? 4ull + 2ull * nx2 + r4(nx2) + r4(l + 1) + sum2 : (uint64_t)l * ncw;
   const bool want_aux = !skip && nC > 0 && aux_words <= P.col_budget;
   const bool want_cols = want_aux && !small;
   uint32_t* cols = aux;
@@ -1327,7 +1740,8 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
     if (want_aux && small) {
       // gx: rows of the X2 vertices, and per universe vertex u_j the list of its X2 neighbours
       unsigned long long* xrow = (unsigned long long*)(gx + 4);
-      uint32_t* coff = gx + 4 + 2 * nx2;
+      uint32_t* xid = gx + 4 + 2 * nx2;
+      uint32_t* coff = xid + r4(nx2);
       uint32_t* cx = coff + r4(l + 1);
       if (lane == 0) {
         gx[0] = nx2;
@@ -1336,10 +1750,15 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
       uint32_t n2 = 0;
       for (uint32_t b = 0; b < nocc; b += 32) {
         const uint32_t x = b + lane;
-        const unsigned long long row = x < nocc ? ldv(vals + occl[x]) : 0ull;
+        const uint32_t slot = x < nocc ? occl[x] : 0u;
+        const unsigned long long row = x < nocc ? ldv(vals + slot) : 0ull;
         const bool is2 = __popcll(row) >= 2;
         const uint32_t bal = __ballot_sync(GMBE_FULL, is2);
-        if (is2) xrow[n2 + __popc(bal & lanemask_lt())] = row;
+        if (is2) {
+          const uint32_t pos = n2 + __popc(bal & lanemask_lt());
+          xrow[pos] = row;
+          xid[pos] = ldv(keys + slot);
+        }
         n2 += __popc(bal);
       }
       __syncwarp();
@@ -1545,6 +1964,7 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
   __shared__ unsigned long long s_tvals[8][kSmemTable ? kSmemTable : 1];
   __shared__ uint32_t s_tkeys[8][kSmemTable ? kSmemTable : 1];
   __shared__ uint32_t s_tocc[8][kSmemTable ? kSmemTable / 2 : 1];
+  __shared__ ThrSmem s_thr[8];
   const uint32_t lane = lane_id();
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   uint32_t* base = P.arena + (uint64_t)gw * P.arena_words;
@@ -1627,7 +2047,7 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       }
     }
     if (kind != 2) {
-      if (top) dispatch_task(P, Tc, top, lo, M.dyn_end, lmap, A, M.sm_sort);
+      if (top) dispatch_task(P, Tc, top, lo, M.dyn_end, lmap, A, M.sm_sort, &s_thr[threadIdx.x >> 5]);
       if (P.timeline) timeline_rec(P, kind, item, g0, tl_info(A.nodes - n0, tl_l, tl_c));
       if (P.per_root_cycles && lane == 0)
         atomicAdd(P.per_root_cycles + item, (unsigned long long)(clock64() - c0));
@@ -1887,6 +2307,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.profile = o.phase_cycles ? 1 : 0;
   P.debug = o.reserved0;
   P.donate = (o.reserved0 & 4) ? 0 : 1;
+  P.thr_min_est = o.reserved1 ? o.reserved1 : GMBE_THR_MIN_EST;
   P.timeline = (unsigned long long*)o.timeline;
   P.timeline_cap = o.timeline_cap;
   if (P.timeline) GMBE_CUDA_TRY(cudaMemsetAsync(P.timeline, 0, 8, s));

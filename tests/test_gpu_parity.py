@@ -295,3 +295,47 @@ def test_full_config_forced_donation(gmbe, name):
         assert (r.nodes, r.nonmax, r.roots_run) == (gd["nodes"], gd["nonmax"], gd["roots_run"])
     finally:
         g.free()
+
+
+# ---------------------------------------------------------------- thread-level tier (run_thr)
+def test_thread_tier_invariance(gmbe, dense_case):
+    """The thread-level subtree tier (one subtree per lane, in-warp donation) and the warp-level tier
+    walk the same canonical tree: identical sets, counts, checksums and counters."""
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        st = g.enumerate(thr_min=1, debug=32, phases=True)
+        ph = list(st.phase_cycles.values())
+        assert ph[1] > 0, "thread tier not exercised"
+        _same(st, o)
+        for kw in (dict(debug=16), dict(thr_min=1), dict(thr_min=1, debug=8), dict(thr_min=1, debug=4),
+                   dict(thr_min=1, bound_height=1, bound_size=1), dict(thr_min=1, warps_per_sm=64),
+                   dict(thr_min=1 << 20)):
+            r = g.enumerate(records=True, **kw)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques), kw
+        o2 = oracle.oracle_mbe(nu, nv, e, prune=False)
+        r = g.enumerate(prune=False, thr_min=1)
+        _same(r, o2)
+    finally:
+        g.free()
+
+
+def test_thread_tier_random(gmbe):
+    """Random dense graphs with planted blocks, every eligible job on the thread tier."""
+    rng = np.random.default_rng(31)
+    for it in range(60):
+        nu, nv = int(rng.integers(8, 70)), int(rng.integers(8, 64))
+        a = rng.random((nu, nv)) < float(rng.uniform(0.05, 0.4))
+        a[: nu // 2, : nv // 3] |= rng.random((nu // 2, nv // 3)) < 0.8
+        e = np.argwhere(a).astype(np.uint32)
+        o = oracle.oracle_mbe(nu, nv, e, records=True)
+        g = gmbe.load(nu, nv, e)
+        try:
+            for kw in (dict(thr_min=1), dict(thr_min=1, debug=8)):
+                r = g.enumerate(records=True, rec_cap=1 << 18, ids_cap=1 << 24, **kw)
+                _same(r, o)
+                if not r.truncated:
+                    assert r.bicliques == sorted(o.bicliques), (it, kw)
+        finally:
+            g.free()
