@@ -95,7 +95,8 @@ typedef struct {
   uint32_t part_index;    /* root shard: enumerate the roots whose degree rank r satisfies */
   uint32_t part_count;    /*   r % part_count == part_index (0 = 1 part); shards partition the
                                output, so counts / checksums add (mod 2^64) across parts */
-  uint32_t reserved0, reserved1;  /* must be 0 */
+  uint32_t reserved0;     /* debug bits for tests / experiments (0 in production use) */
+  uint32_t reserved1;     /* must be 0 */
   /* Optional bounded output (device-accessible memory: device or mapped pinned host).
    * Record = [|L|, |R|, L ids (caller U ids), R ids (caller V ids)], order within a record and of
    * records unspecified; out_offsets[i] = word offset of record i in out_ids.  A full buffer is
@@ -127,6 +128,14 @@ typedef struct {
   uint64_t pool_words;
   uint64_t queue_cap;
   void* cuda_stream;      /* NULL = the graph's stream */
+  /* B200 scheduling knobs (0 = default; both leave the result and the canonical-tree counters
+   * unchanged): */
+  uint32_t split_wide;    /* also split a task over a wide universe (|L| > 64 bits) when
+                             |C|·⌈|L|/32⌉ >= split_wide (default 32): such nodes cost ~|L|/32 words
+                             each, so even small subtrees are worth spreading over warps */
+  uint32_t thr_min;       /* thread-level tier: jobs (<= 32 candidates over <= 64 universe bits)
+                             with Σ_c (|N(c) ∩ L| - 1) >= thr_min run one subtree per lane
+                             (default 16; UINT32_MAX disables the tier) */
 } gmbe_opts;
 
 typedef struct {

@@ -51,7 +51,8 @@ class Opts(ctypes.Structure):
                 ("out_offsets", _vp), ("out_offsets_cap", _u64), ("out_ids", _vp),
                 ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("phase_cycles", _vp), ("timeline", _vp), ("timeline_cap", _u64),
                 ("arena_words", _u64),
-                ("pool_words", _u64), ("queue_cap", _u64), ("cuda_stream", _vp)]
+                ("pool_words", _u64), ("queue_cap", _u64), ("cuda_stream", _vp),
+                ("split_wide", _u32), ("thr_min", _u32)]
 
 
 class CResult(ctypes.Structure):
@@ -150,7 +151,7 @@ class Graph:
 
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
-                  per_root=False, root_cycles=False, phases=False, timeline=0, debug=0, thr_min=0, arena_words=0, pool_words=0, queue_cap=0, stream=None):
+                  per_root=False, root_cycles=False, phases=False, timeline=0, debug=0, thr_min=0, split_wide=0, arena_words=0, pool_words=0, queue_cap=0, stream=None):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
@@ -161,7 +162,7 @@ class Graph:
         o.arena_words, o.pool_words, o.queue_cap = arena_words, pool_words, queue_cap
         o.cuda_stream = _stream_ptr(stream)
         o.reserved0 = debug
-        o.reserved1 = thr_min  # experiments: run_thr tier threshold (0 = built-in)
+        o.thr_min, o.split_wide = thr_min, split_wide
         bufs = None
         if records:
             import torch

@@ -26,6 +26,8 @@
 #include <string>
 #include <vector>
 
+#include <cub/cub.cuh>
+
 #include "gmbe_internal.cuh"
 
 namespace {
@@ -57,6 +59,7 @@ enum : unsigned int { kErrArena = 1 };
 struct Params {
   DevGraph g;
   uint32_t n_roots;  // roots of this shard
+  const uint32_t* issue;  // the shard's roots (ranks) in issue order: most wedges first
   uint32_t part_index, part_count;
   uint32_t prune, split, bound_height, bound_size;
   uint32_t hu_side;   // checksum side of the library's U vertices (0 = caller U)
@@ -79,9 +82,11 @@ struct Params {
   unsigned long long* per_root_cycles;
   uint32_t profile;
   uint32_t debug;  // opts.reserved0 bits (tests / experiments): 4 = no donation, 8 = donate whenever possible,
-                   // 16 = no thread-level tier (run_thr), 32 = path statistics into ctrl.phase
+                   // 16 = no thread-level tier (run_thr), 32 = path statistics into ctrl.phase,
+                   // 64 = no suffix-mode roots, 128 = every root in suffix mode
   uint32_t donate;  // dynamic donation to idle warps (donate_reg)
-  uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.reserved1 overrides; experiments)
+  uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.thr_min)
+  uint32_t split_wide;   // wide-universe split threshold on |C|·⌈|L|/32⌉ (opts.split_wide)
   unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1, info]*
   uint64_t timeline_cap;
 };
@@ -268,10 +273,23 @@ __device__ __forceinline__ uint32_t ht_find(const uint32_t* keys, uint32_t shift
   }
 }
 
+// first position in the rank-sorted list a[0, n) holding a rank > r
+__device__ __forceinline__ uint32_t upper_rank(const uint32_t* a, uint32_t n, uint32_t r) {
+  uint32_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (__ldg(a + mid) <= r) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
 // Visit every wedge (i, v): u_i = L[i], v ∈ N(u_i), load-balanced across the warp.
-// f(i, v, active) is called by all 32 lanes each step.
+// f(i, v, active) is called by all 32 lanes each step.  after != kNone: only the wedges to ranks
+// > after (a suffix of each rank-sorted list).
 template <class F>
-__device__ __forceinline__ void for_each_wedge(const DevGraph& g, const uint32_t* L, uint32_t l, F f) {
+__device__ __forceinline__ void for_each_wedge(const DevGraph& g, const uint32_t* L, uint32_t l, F f,
+                                               uint32_t after = 0xffffffffu) {
   const uint32_t lane = lane_id();
   for (uint32_t b = 0; b < l; b += 32) {
     uint32_t i = b + lane, beg = 0, deg = 0;
@@ -279,6 +297,11 @@ __device__ __forceinline__ void for_each_wedge(const DevGraph& g, const uint32_t
       const uint32_t u = L[i];
       beg = g.off_u[u];
       deg = g.off_u[u + 1] - beg;
+      if (after != 0xffffffffu) {
+        const uint32_t s = upper_rank(g.adj_u + beg, deg, after);
+        beg += s;
+        deg -= s;
+      }
     }
     uint32_t inc = deg;
 #pragma unroll
@@ -928,8 +951,15 @@ __device__ __forceinline__ uint32_t rec_words(const TaskCtx& T, const uint32_t* 
   return kHdr + T.W4 + rec[0] * T.E;
 }
 __device__ __forceinline__ bool heavy(const Params& P, uint32_t l, uint32_t nC) {
+  if (!P.split) return false;
   const unsigned long long h = min(l, nC);  // tree height estimate
-  return P.split && h > P.bound_height && h * nC > P.bound_size;
+  if (h > P.bound_height && h * nC > P.bound_size) return true;
+  // wide universes: every node costs ~|L|/32 words of AND/POPC plus a Γ test over |L'| members, so
+  // the node count alone under-estimates the work (B200 addition, reading B4)
+  return l > 64 && nC >= 2 && (unsigned long long)nC * ((l + 31) / 32) >= P.split_wide;
+}
+__device__ __forceinline__ bool heavy_wide(const Params& P, uint32_t l, uint32_t nC) {
+  return P.split && l > 64 && nC >= 2 && (unsigned long long)nC * ((l + 31) / 32) >= P.split_wide;
 }
 
 // Walk the subtree of `top` (Alg 2) on the node stack [stack_lo, stack_hi) -- or, when the task is
@@ -1251,6 +1281,9 @@ __device__ bool donate_thr(const Params& P, const TaskCtx& T, uint32_t lmap, Acc
 
 #ifndef GMBE_NI_THR
 #define GMBE_NI_THR 0
+#endif
+#ifndef GMBE_SPLIT_WIDE
+#define GMBE_SPLIT_WIDE 32
 #endif
 #ifndef GMBE_THR_MIN_EST
 #define GMBE_THR_MIN_EST 16  // jobs with fewer adjacency bits (Σ(k-1)) stay on run_reg (setup > work)
@@ -1595,8 +1628,9 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     int r;
     if constexpr (LPE == 0) r = gen_child_small(P, T, cur, i, ch, A, smem);
     else r = gen_child<LPE>(P, T, cur, i, ch, A, smem);
-    if (r == 2 && split_mode && cur == top) {
-      // Alg 4 L25: hand the child to the task queue as a self-contained subtask
+    // Alg 4 L25: hand the child to the task queue as a self-contained subtask -- every child of a
+    // heavy top, and (wide universes) any child that is itself heavy (reading B4)
+    if (r == 2 && ((split_mode && cur == top) || (LPE != 0 && heavy_wide(P, lmap, ch[0])))) {
       PH_START(A);
       const bool done = task_publish(P, T, lmap, T.rlist ? ch[5] : 0, ch, rec_words(T, ch), A);
       PH_STOP(A, 7);
@@ -1634,6 +1668,47 @@ __device__ GMBE_NI_IF(GMBE_NI_DISPATCH) void dispatch_task(const Params& P, Task
 }
 
 // ---------------------------------------------------------------- root task (a3)
+// Alg 3 L7 for a root scanned in suffix mode (below): is some vertex ranked before v_s adjacent to
+// all of L_r?  Such a vertex x lies in N(u*) for the lowest-degree u* ∈ L_r, below rank r in its
+// rank-sorted list, and has deg(x) >= |L_r|; each survivor of that filter is tested warp-wide by
+// binary searches of the members of L_r in the sorted list N(x) (first miss ends the test).
+__device__ bool earlier_dominator(const DevGraph& g, const uint32_t* Lr, uint32_t l, uint32_t r) {
+  const uint32_t lane = lane_id();
+  unsigned long long key = ~0ull;
+  for (uint32_t j = lane; j < l; j += 32) {
+    const uint32_t u = Lr[j];
+    key = min(key, ((unsigned long long)(g.off_u[u + 1] - g.off_u[u]) << 32) | j);
+  }
+  for (int o = 16; o; o >>= 1) key = min(key, (unsigned long long)__shfl_xor_sync(GMBE_FULL, key, o));
+  const uint32_t us = Lr[(uint32_t)key];
+  const uint32_t* a = g.adj_u + g.off_u[us];
+  const uint32_t n = r ? upper_rank(a, (uint32_t)(key >> 32), r - 1) : 0u;  // ranks < r
+  for (uint32_t b = 0; b < n; b += 32) {
+    const uint32_t x = b + lane < n ? __ldg(a + b + lane) : kNone;
+    uint32_t xb = 0, xd = 0;
+    if (x != kNone) {
+      xb = g.off_v[x];
+      xd = g.off_v[x + 1] - xb;
+    }
+    uint32_t cand = __ballot_sync(GMBE_FULL, x != kNone && xd >= l);
+    while (cand) {
+      const uint32_t src = __ffs(cand) - 1;
+      cand &= cand - 1;
+      const uint32_t cb = __shfl_sync(GMBE_FULL, xb, src), cd = __shfl_sync(GMBE_FULL, xd, src);
+      bool all = true;
+      for (uint32_t base = 0; base < l && all; base += 32) {
+        const uint32_t j = base + lane;
+        all = __all_sync(GMBE_FULL, j >= l || bsearch_rank(g.adj_v + cb, cd, Lr[j]));
+      }
+      if (all) return true;
+    }
+  }
+  return false;
+}
+#ifndef GMBE_SUFFIX_MIN
+#define GMBE_SUFFIX_MIN 8192  // roots with at least this many wedges may scan only later ranks
+#endif
+
 // Root v_s (rank r): L_r = N(v_s); wedge scan of N2(v_s) with k(v) = |N(v) ∩ L_r|.  Emits the root
 // biclique and, if it has candidates, prepares its node record as a task (Tc, *top, stack from *lo)
 // for the caller's single dispatch site; returns whether it did.
@@ -1651,8 +1726,35 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   }
   const uint32_t wedges = warp_sum(wp);
   A.abytes += 4ull * (l + wedges);
-  const uint32_t T = next_pow2(max(64u, 2u * wedges));
-  if (T > P.tmax || wedges > P.omax) {
+  // Suffix mode (B200 addition, reading B5): a root with many wedges but few of them to
+  // later-ranked vertices (high degree rank: few candidates, huge excluded set) counts k only over
+  // the rank suffix of each list; the skip test (Alg 3 L7) then looks for an earlier dominator
+  // directly, and the children test maximality without a Γ index (gamma_is_r).
+  uint32_t after = kNone, scanned = wedges;
+  if (P.debug & 128) {  // tests: every root in suffix mode
+    after = r;
+  } else if (wedges >= GMBE_SUFFIX_MIN && !(P.debug & 64)) {
+    uint32_t sp = 0;
+    for (uint32_t j = lane; j < l; j += 32) {
+      const uint32_t u = Lr[j], ub = g.off_u[u], du = g.off_u[u + 1] - ub;
+      sp += du - upper_rank(g.adj_u + ub, du, r);
+    }
+    sp = warp_sum(sp);
+    if (4ull * sp < wedges) {
+      after = r;
+      scanned = sp;
+    }
+  }
+  if (after != kNone && (P.debug & 128)) {
+    uint32_t sp = 0;
+    for (uint32_t j = lane; j < l; j += 32) {
+      const uint32_t u = Lr[j], ub = g.off_u[u], du = g.off_u[u + 1] - ub;
+      sp += du - upper_rank(g.adj_u + ub, du, r);
+    }
+    scanned = warp_sum(sp);
+  }
+  const uint32_t T = next_pow2(max(64u, 2u * scanned));
+  if (T > P.tmax || scanned > P.omax) {
     if (lane == 0) atomicOr(&P.ctrl->error, kErrArena);
     return false;
   }
@@ -1672,7 +1774,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
       if (small) atomicOr(vals + h, 1ull << i);
       else atomicAdd(vals + h, 1ull);
     }
-  });
+  }, after);
   __syncwarp();
   PH_STOP(A, 0);
   // classify: k == |L| -> R (root skipped unless v_s is the earliest vertex of R, Alg 3 L7);
@@ -1708,6 +1810,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
     nC += __popc(bC);
   }
   skip = __any_sync(GMBE_FULL, skip);
+  if (after != kNone && !skip && sort_fits) skip = earlier_dominator(g, Lr, l, r);
   sum2 = warp_sum(sum2);
   PH_STOP(A, 1);
   // Γ index over X2 = {x in the 2-hop set X : |N(x) ∩ L_r| >= 2} (the maximality test of an L' with
@@ -1716,7 +1819,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   const uint32_t ncw = (nx2 + 31) / 32;
   uint32_t* aux = align4((uint32_t*)(sortbuf + next_pow2(max(nC, 1u))));
   const uint64_t aux_words = small ? 4ull + 2ull * nx2 + r4(nx2) + r4(l + 1) + sum2 : (uint64_t)l * ncw;
-  const bool want_aux = !skip && nC > 0 && aux_words <= P.col_budget;
+  const bool want_aux = !skip && nC > 0 && after == kNone && aux_words <= P.col_budget;
   const bool want_cols = want_aux && !small;
   uint32_t* cols = aux;
   uint32_t* gx = aux;
@@ -1869,7 +1972,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
             if (want_cols && xi) atomicOr(cols + (size_t)i * ncw + ((xi - 1) >> 5), 1u << ((xi - 1) & 31));
             if (x & 0x80000000ull) atomicOr(ent + (size_t)(x & 0x7fffffffull) * E + (i >> 5), 1u << (i & 31));
           }
-        });
+        }, after);
         __syncwarp();
         __threadfence();  // rows / columns were built with atomics: drop stale L1 lines
       }
@@ -2036,7 +2139,7 @@ __global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
       }
       t = __shfl_sync(GMBE_FULL, t, 0);
       if (t < P.n_roots) {
-        const uint32_t rk = P.part_index + (P.n_roots - 1 - (uint32_t)t) * P.part_count;
+        const uint32_t rk = P.issue[t];
         kind = 0;
         item = rk;
         if (run_root(P, rk, M, A, Tc, &top, &lo)) lmap = top[2];
@@ -2109,6 +2212,14 @@ struct Workspace {
   size_t per_root_bytes = 0;
   void* per_root_cyc = nullptr;
   size_t per_root_cyc_bytes = 0;
+  void* shard = nullptr;  // this call's root issue list (part_count > 1) + selection scratch
+  size_t shard_bytes = 0;
+};
+
+// roots of one shard (rank % part_count == part_index), kept in the graph's issue order
+struct ShardOf {
+  uint32_t pc, pi;
+  __host__ __device__ __forceinline__ bool operator()(const uint32_t& r) const { return r % pc == pi; }
 };
 
 cudaError_t ensure(void** p, size_t* have, size_t need) {
@@ -2159,7 +2270,7 @@ extern "C" void gmbe_release_workspace(const gmbe_graph* G) {
       i++;
       continue;
     }
-    for (void* p : {w->arena, w->pool, w->rings, w->rbuf, w->ctrl, w->per_root, w->per_root_cyc})
+    for (void* p : {w->arena, w->pool, w->rings, w->rbuf, w->ctrl, w->per_root, w->per_root_cyc, w->shard})
       if (p) cudaFree(p);
     delete w;
     g_ws_idle.erase(g_ws_idle.begin() + i);
@@ -2280,6 +2391,18 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.part_index = o.part_index;
   P.part_count = parts;
   P.n_roots = g.n_v > o.part_index ? (g.n_v - o.part_index + parts - 1) / parts : 0;
+  P.issue = g.issue;
+  if (parts > 1 && P.n_roots) {
+    size_t tb = 0;
+    GMBE_CUDA_TRY(cub::DeviceSelect::If(nullptr, tb, g.issue, (uint32_t*)nullptr, (int*)nullptr, (int)g.n_v,
+                                        ShardOf{parts, o.part_index}, s));
+    const size_t list_b = ((size_t)g.n_v * 4 + 255) & ~(size_t)255;
+    GMBE_CUDA_TRY(ensure(&W.shard, &W.shard_bytes, list_b + 256 + tb));
+    char* sb = (char*)W.shard;
+    GMBE_CUDA_TRY(cub::DeviceSelect::If(sb + list_b + 256, tb, g.issue, (uint32_t*)sb, (int*)(sb + list_b),
+                                        (int)g.n_v, ShardOf{parts, o.part_index}, s));
+    P.issue = (const uint32_t*)sb;
+  }
   P.prune = o.no_prune ? 0 : 1;
   P.split = o.no_split ? 0 : 1;
   P.bound_height = o.bound_height ? o.bound_height : 8;    // paper: 20; retuned for B200
@@ -2307,7 +2430,8 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.profile = o.phase_cycles ? 1 : 0;
   P.debug = o.reserved0;
   P.donate = (o.reserved0 & 4) ? 0 : 1;
-  P.thr_min_est = o.reserved1 ? o.reserved1 : GMBE_THR_MIN_EST;
+  P.thr_min_est = o.thr_min ? o.thr_min : GMBE_THR_MIN_EST;
+  P.split_wide = o.split_wide ? o.split_wide : GMBE_SPLIT_WIDE;
   P.timeline = (unsigned long long*)o.timeline;
   P.timeline_cap = o.timeline_cap;
   if (P.timeline) GMBE_CUDA_TRY(cudaMemsetAsync(P.timeline, 0, 8, s));

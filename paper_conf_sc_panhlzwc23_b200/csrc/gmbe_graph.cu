@@ -83,10 +83,15 @@ __global__ void k_low32(const unsigned long long* __restrict__ k, uint64_t m, ui
 }
 
 // one warp per V rank: wedge count Σ_{u∈N(v)} |N(u)| and the maxima.
+__global__ void k_issue(const unsigned long long* __restrict__ keys, uint32_t n, uint32_t* __restrict__ issue) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+    issue[i] = ~(uint32_t)keys[i];
+}
+
 __global__ void k_bounds(const uint32_t* __restrict__ off_v, const uint32_t* __restrict__ adj_v,
                          const uint32_t* __restrict__ off_u, uint32_t n_v, uint32_t n_u,
                          uint32_t* __restrict__ maxes /* [0]=Δ(V) [1]=Δ(U) [2]=wedge bound */,
-                         unsigned long long* __restrict__ rec_bound) {
+                         unsigned long long* __restrict__ rec_bound, unsigned long long* __restrict__ cost_key) {
   uint32_t lane = threadIdx.x & 31;
   uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   uint32_t nw = (gridDim.x * blockDim.x) >> 5;
@@ -99,6 +104,9 @@ __global__ void k_bounds(const uint32_t* __restrict__ off_v, const uint32_t* __r
     }
     for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(GMBE_FULL, s, o);
     if (lane == 0) {
+      // issue key: wedges descending, then rank descending (ascending sort of the complements)
+      const uint32_t w = (uint32_t)(s > 0xffffffffull ? 0xffffffffull : s);
+      cost_key[r] = ((unsigned long long)(~w) << 32) | (~r);
       atomicMax(&maxes[0], e - b);
       atomicMax(&maxes[2], (uint32_t)(s > 0xffffffffull ? 0xffffffffull : s));
       // root record: <= s candidates, each row of ceil(deg/32) words + id + k, padded to 4
@@ -313,7 +321,16 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
     TRY(radix_sort(t, ku, keys2, m, 32 + bits_for(NU), s));
     k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_u), gmbe_note_launch();
   }
-  if (NV || NU) k_bounds<<<grid_for((uint64_t)NV * 32 + NU), 256, 0, s>>>(off_v, adj_v, off_u, NV, NU, maxes, d_recb), gmbe_note_launch();
+  uint32_t* issue;
+  TRY(t.alloc(&issue, NV + 1));
+  unsigned long long *ck, *ck2;
+  TRY(t.alloc(&ck, NV + 1));
+  TRY(t.alloc(&ck2, NV + 1));
+  if (NV || NU) k_bounds<<<grid_for((uint64_t)NV * 32 + NU), 256, 0, s>>>(off_v, adj_v, off_u, NV, NU, maxes, d_recb, ck), gmbe_note_launch();
+  TRY(cudaGetLastError());
+  // root issue order: most wedges first (the schedule only; the tree is fixed by the rank order)
+  TRY(radix_sort(t, ck, ck2, NV, 64, s));
+  if (NV) k_issue<<<grid_for(NV), 256, 0, s>>>(ck2, NV, issue), gmbe_note_launch();
   TRY(cudaGetLastError());
   uint32_t hm[4];
   TRY(cudaMemcpyAsync(hm, maxes, sizeof(hm), cudaMemcpyDeviceToHost, s));
@@ -321,7 +338,7 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   TRY(cudaMemcpyAsync(&h_recb, d_recb, 8, cudaMemcpyDeviceToHost, s));
   TRY(cudaStreamSynchronize(s));
 
-  void* keep[] = {off_v, adj_v, off_u, adj_u, rank2id, hv};
+  void* keep[] = {off_v, adj_v, off_u, adj_u, rank2id, hv, issue};
   for (void* q : keep) {
     t.release(q);
     G->bufs[G->nbufs++] = q;
@@ -337,6 +354,7 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   g.adj_u = adj_u;
   g.rank2id = rank2id;
   g.hv = hv;
+  g.issue = issue;
   g.delta_v = hm[0];
   g.delta_u = hm[1];
   g.wedge_bound = hm[2];

@@ -23,6 +23,7 @@ struct DevGraph {
   const uint32_t* adj_u;    // [m]      v ranks, ascending
   const uint32_t* rank2id;  // [n_v]    rank -> id on the library's V side (== caller id of that side)
   const unsigned long long* hv;  // [n_v] checksum hash of each V vertex by rank (caller roles)
+  const uint32_t* issue;    // [n_v]    ranks by wedges descending: the root issue order (schedule only)
   uint32_t delta_u, delta_v, wedge_bound;  // wedge_bound = max_v Σ_{u∈N(v)} |N(u)|
   uint64_t rec_bound;  // max_v wedges(v) * entry stride(|N(v)|): bound on a root node record (words)
 };

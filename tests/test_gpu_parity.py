@@ -339,3 +339,44 @@ def test_thread_tier_random(gmbe):
                     assert r.bicliques == sorted(o.bicliques), (it, kw)
         finally:
             g.free()
+
+
+def test_suffix_mode_roots(gmbe, dense_case):
+    """Suffix-mode roots (k counted over later ranks only, Alg 3 L7 by an earlier-dominator search,
+    no Γ index; reading B5) give the canonical tree: forced on every root (debug 128)."""
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        for kw in (dict(debug=128), dict(debug=128 | 16), dict(debug=128, bound_height=1, bound_size=1)):
+            r = g.enumerate(records=True, **kw)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques), kw
+    finally:
+        g.free()
+    rng = np.random.default_rng(77)
+    for it in range(80):
+        nu, nv, e = _rand_graph(rng, nmax=14)
+        o = oracle.oracle_mbe(nu, nv, e, records=True)
+        r = _run(gmbe, nu, nv, e, records=True, debug=128)
+        _same(r, o)
+        assert r.bicliques == sorted(o.bicliques)
+
+
+def test_wide_universe_splitting(gmbe):
+    """Universes above 64 bits (W > 2 words per row) with the wide-universe split rule forced on
+    every node with >= 2 candidates (split_wide=1): same tree, counters and sets."""
+    rng = np.random.default_rng(123)
+    for it in range(12):
+        nu, nv = int(rng.integers(120, 260)), int(rng.integers(20, 45))
+        a = rng.random((nu, nv)) < float(rng.uniform(0.25, 0.5))
+        e = np.argwhere(a).astype(np.uint32)
+        o = oracle.oracle_mbe(nu, nv, e, records=True)
+        g = gmbe.load(nu, nv, e)
+        try:
+            for kw in (dict(split_wide=1), dict(split_wide=1, debug=128), dict(split_wide=1 << 30)):
+                r = g.enumerate(records=True, rec_cap=1 << 18, ids_cap=1 << 24, **kw)
+                _same(r, o)
+                if not r.truncated:
+                    assert r.bicliques == sorted(o.bicliques), (it, kw)
+        finally:
+            g.free()
