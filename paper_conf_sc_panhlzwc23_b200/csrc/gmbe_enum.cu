@@ -365,8 +365,55 @@ __device__ __forceinline__ unsigned long long warp_sort32(unsigned long long x) 
   }
   return x;
 }
-// sort n keys in a[0..n) (room for next_pow2(n))
-__device__ void warp_sort_keys(unsigned long long* a, uint32_t n, unsigned long long* smem) {
+// one stable LSD radix pass by one warp: dst = src sorted by bits [shift, shift + dbits) (dbits <= 8),
+// histogram in shared memory (hist: 256 words)
+__device__ void warp_radix_pass(const unsigned long long* src, unsigned long long* dst, uint32_t n, uint32_t shift,
+                                uint32_t dbits, uint32_t* hist) {
+  const uint32_t lane = lane_id(), nb = 1u << dbits;
+  for (uint32_t i = lane; i < nb; i += 32) hist[i] = 0;
+  __syncwarp();
+  for (uint32_t b = 0; b < n; b += 32) {
+    const uint32_t j = b + lane;
+    const uint32_t d = j < n ? (uint32_t)(src[j] >> shift) & (nb - 1) : nb;
+    const uint32_t peers = __match_any_sync(GMBE_FULL, d);
+    if (j < n && lane == __ffs(peers) - 1) hist[d] += __popc(peers);
+    __syncwarp();
+  }
+  // exclusive scan of hist (lane t owns the nb/32 consecutive entries of chunk t)
+  const uint32_t per = (nb + 31) / 32;
+  uint32_t loc = 0;
+  for (uint32_t k = 0; k < per; k++)
+    if (lane * per + k < nb) loc += hist[lane * per + k];
+  uint32_t inc = loc;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t t = __shfl_up_sync(GMBE_FULL, inc, o);
+    if (lane >= (uint32_t)o) inc += t;
+  }
+  uint32_t run = inc - loc;
+  __syncwarp();
+  for (uint32_t k = 0; k < per; k++)
+    if (lane * per + k < nb) {
+      const uint32_t c = hist[lane * per + k];
+      hist[lane * per + k] = run;
+      run += c;
+    }
+  __syncwarp();
+  for (uint32_t b = 0; b < n; b += 32) {
+    const uint32_t j = b + lane;
+    const unsigned long long x = j < n ? src[j] : 0ull;
+    const uint32_t d = j < n ? (uint32_t)(x >> shift) & (nb - 1) : nb;
+    const uint32_t peers = __match_any_sync(GMBE_FULL, d);
+    if (j < n) dst[hist[d] + __popc(peers & lanemask_lt())] = x;
+    __syncwarp();
+    if (j < n && lane == __ffs(peers) - 1) hist[d] += __popc(peers);
+    __syncwarp();
+  }
+}
+// sort n keys in a[0..n) (room for next_pow2(n)); keys above kSmemSort with a scratch tmp[0..n)
+// and key_bits (significant high bits, keys compared on [64 - key_bits, 64) and then low bits
+// irrelevant -- the callers' keys are unique in their high part) use an LSD radix sort
+__device__ void warp_sort_keys(unsigned long long* a, uint32_t n, unsigned long long* smem,
+                               unsigned long long* tmp = nullptr, uint32_t hi_bits = 0) {
   const uint32_t lane = lane_id();
   if (n <= 1) return;
   if (n <= 32) {
@@ -382,6 +429,12 @@ __device__ void warp_sort_keys(unsigned long long* a, uint32_t n, unsigned long 
     warp_bitonic64(smem, n);
     for (uint32_t j = lane; j < n; j += 32) a[j] = smem[j];
     __syncwarp();
+    return;
+  }
+  if (smem && tmp && hi_bits) {  // keys = (unique value < 2^hi_bits) << 32 | payload
+    const uint32_t passes = hi_bits <= 16 ? 2u : 4u, dbits = (hi_bits + passes - 1) / passes;
+    for (uint32_t p = 0; p < passes; p++)
+      warp_radix_pass(p & 1 ? tmp : a, p & 1 ? a : tmp, n, 32 + p * dbits, dbits, (uint32_t*)smem);
     return;
   }
   warp_bitonic64(a, n);
@@ -1924,7 +1977,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
       // root node record: candidates in rank order (Alg 2 L6 "smallest first")
       __syncwarp();
       PH_STOP(A, 3);
-      warp_sort_keys(sortbuf, nC, M.sm_sort);
+      warp_sort_keys(sortbuf, nC, M.sm_sort, (unsigned long long*)rec, 32 - __clz(max(g.n_v, 2u) - 1));
       PH_STOP(A, 2);
       uint32_t* ent = rec + kHdr + W4;
       for (uint32_t j = lane; j < nC; j += 32) {
