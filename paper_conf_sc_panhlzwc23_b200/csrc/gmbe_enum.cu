@@ -83,7 +83,8 @@ struct Params {
   uint32_t profile;
   uint32_t debug;  // opts.reserved0 bits (tests / experiments): 4 = no donation, 8 = donate whenever possible,
                    // 16 = no thread-level tier (run_thr), 32 = path statistics into ctrl.phase,
-                   // 64 = no suffix-mode roots, 128 = every root in suffix mode
+                   // 64 = no suffix-mode roots, 128 = every root in suffix mode, 256 = no dense-mode roots,
+                   // 512 = dense mode whenever the table can hold it
   uint32_t donate;  // dynamic donation to idle warps (donate_reg)
   uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.thr_min)
   uint32_t split_wide;   // wide-universe split threshold on |C|·⌈|L|/32⌉ (opts.split_wide)
@@ -1465,6 +1466,7 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
   unsigned long long L = L0, SR = ((unsigned long long)rec[7] << 32) | rec[6];
   const uint32_t cand_all = nC >= 32 ? GMBE_FULL : ((1u << nC) - 1u);
   uint32_t C = cand_all, next = 0, Rm = 0, d = 0, dmask = 0;
+  uint32_t bd = 0;  // tree depth (below the job's top) of this lane's level 0
   uint32_t n_nodes = 0, n_nonmax = 0, n_count = 0;
   unsigned long long abytes = 0, cks = 0;
 #if GMBE_DONATE
@@ -1489,48 +1491,15 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     }
     const uint32_t idle = __ballot_sync(GMBE_FULL, !has);
     if (idle == GMBE_FULL) break;
-    if (idle) {  // in-warp donation: the r-th idle lane takes the shallowest level of the r-th donor
-      const uint32_t donors = __ballot_sync(GMBE_FULL, dmask != 0);
-      if (donors) {
-        const uint32_t nd = min(__popc(idle), __popc(donors));
-        unsigned long long gL = 0, gSR = 0;
-        uint32_t gC = 0, gRm = 0, gnext = 0;
-        if (dmask && __popc(donors & lanemask_lt()) < nd) {
-          const uint32_t k = __ffs(dmask) - 1;
-          gL = stk[k].L;
-          gSR = stk[k].SR;
-          gC = stk[k].C;
-          gRm = stk[k].Rm;
-          gnext = stk[k].next;
-          stk[k].next = 32;  // the remaining children of level k are no longer this lane's
-          dmask &= ~(1u << k);
-        }
-        const uint32_t ir = __popc(idle & lanemask_lt());
-        const bool take = !has && ir < nd;
-        const uint32_t src = take ? __fns(donors, 0, ir + 1) : lane;
-        gL = shfl64(gL, src);
-        gSR = shfl64(gSR, src);
-        gC = __shfl_sync(GMBE_FULL, gC, src);
-        gRm = __shfl_sync(GMBE_FULL, gRm, src);
-        gnext = __shfl_sync(GMBE_FULL, gnext, src);
-        if (take) {
-          has = true;
-          L = gL;
-          SR = gSR;
-          C = gC;
-          Rm = gRm;
-          next = gnext;
-          d = 0;
-          dmask = 0;
-        }
-      }
-    }
 #if GMBE_DONATE
-    if ((!idle || (P.debug & 8)) && P.donate && (++tick & 7) == 0 && hungry(P)) {  // cross-warp donation to idle warps
-      const uint32_t donors = __ballot_sync(GMBE_FULL, dmask != 0);
-      if (donors) {
-        const uint32_t src = __ffs(donors) - 1;
-        const uint32_t k = lane == src ? __ffs(dmask) - 1 : 0;
+    if (P.donate && (++tick & 3) == 0 && hungry(P)) {  // cross-warp donation to idle warps
+      // the donor: the lane whose shallowest stacked level with untraversed children is the
+      // shallowest in the job's tree (the largest piece of remaining work)
+      const uint32_t key =
+          __reduce_min_sync(GMBE_FULL, dmask ? ((bd + (uint32_t)(__ffs(dmask) - 1)) << 5) | lane : kNone);
+      if (key != kNone) {
+        const uint32_t src = key & 31u;
+        const uint32_t k = lane == src ? (uint32_t)(__ffs(dmask) - 1) : 0u;
         unsigned long long kL = 0, kSR = 0;
         uint32_t kC = 0, kRm = 0, knext = 0;
         if (lane == src) {
@@ -1548,6 +1517,45 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
       }
     }
 #endif
+    if (idle) {  // in-warp donation: the r-th idle lane takes the shallowest level of the r-th donor
+      const uint32_t donors = __ballot_sync(GMBE_FULL, dmask != 0);
+      if (donors) {
+        const uint32_t nd = min(__popc(idle), __popc(donors));
+        unsigned long long gL = 0, gSR = 0;
+        uint32_t gC = 0, gRm = 0, gnext = 0, gbd = 0;
+        if (dmask && __popc(donors & lanemask_lt()) < nd) {
+          const uint32_t k = __ffs(dmask) - 1;
+          gbd = bd + k;
+          gL = stk[k].L;
+          gSR = stk[k].SR;
+          gC = stk[k].C;
+          gRm = stk[k].Rm;
+          gnext = stk[k].next;
+          stk[k].next = 32;  // the remaining children of level k are no longer this lane's
+          dmask &= ~(1u << k);
+        }
+        const uint32_t ir = __popc(idle & lanemask_lt());
+        const bool take = !has && ir < nd;
+        const uint32_t src = take ? __fns(donors, 0, ir + 1) : lane;
+        gL = shfl64(gL, src);
+        gSR = shfl64(gSR, src);
+        gC = __shfl_sync(GMBE_FULL, gC, src);
+        gRm = __shfl_sync(GMBE_FULL, gRm, src);
+        gnext = __shfl_sync(GMBE_FULL, gnext, src);
+        gbd = __shfl_sync(GMBE_FULL, gbd, src);
+        if (take) {
+          has = true;
+          bd = gbd;
+          L = gL;
+          SR = gSR;
+          C = gC;
+          Rm = gRm;
+          next = gnext;
+          d = 0;
+          dmask = 0;
+        }
+      }
+    }
     if (!has) continue;
     // generate the child via the next candidate i (Alg 2 L6-13)
     const uint32_t i = __ffs(C & (GMBE_FULL << next)) - 1;
@@ -1817,18 +1825,50 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   unsigned long long* vals = stab ? M.svals : M.vals;
   uint32_t* occl = stab ? M.socc : M.occ;
   const bool small = l <= 64;  // rows (<= 64 bits) straight from the table
+  // Dense mode (heavy roots): the warp's table values indexed by rank directly (n_v <= table
+  // slots).  Pass 1 is then fire-and-forget atomics (no probing), and the occupied list comes from
+  // a scan of the rank range -- in rank order, so the candidates need no sort.
+  const uint32_t lo_v = after != kNone ? r + 1 : 0u;
+  const bool dense = !stab && g.n_v <= P.tmax && !(P.debug & 256) &&
+                     ((uint64_t)(g.n_v - lo_v) <= 16ull * scanned || (P.debug & 512));
   PH_START(A);
   // pass 1 (Alg 3 L2-3)
   uint32_t nocc = 0;
-  for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
-    const bool a = act && v != r;
-    const uint32_t h = ht_insert_warp(keys, shift, mask, v, a, occl, nocc);
-    if (a) {
-      if (small) atomicOr(vals + h, 1ull << i);
-      else atomicAdd(vals + h, 1ull);
+  if (dense) {
+    for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
+      if (act && v != r) {
+        if (small) atomicOr(vals + v, 1ull << i);
+        else atomicAdd(vals + v, 1ull);
+      }
+    }, after);
+    __syncwarp();
+    __threadfence();
+    for (uint32_t b = lo_v; b < g.n_v; b += 256) {
+      unsigned long long x[8];
+#pragma unroll
+      for (int q = 0; q < 8; q++) {
+        const uint32_t v = b + q * 32 + lane;
+        x[q] = v < g.n_v ? __ldcg(vals + v) : 0ull;  // L2: pass 1 wrote with atomics
+      }
+#pragma unroll
+      for (int q = 0; q < 8; q++) {
+        const uint32_t bal = __ballot_sync(GMBE_FULL, x[q] != 0ull);
+        if (x[q]) occl[nocc + __popc(bal & lanemask_lt())] = b + q * 32 + lane;
+        nocc += __popc(bal);
+      }
     }
-  }, after);
-  __syncwarp();
+    __syncwarp();
+  } else {
+    for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
+      const bool a = act && v != r;
+      const uint32_t h = ht_insert_warp(keys, shift, mask, v, a, occl, nocc);
+      if (a) {
+        if (small) atomicOr(vals + h, 1ull << i);
+        else atomicAdd(vals + h, 1ull);
+      }
+    }, after);
+    __syncwarp();
+  }
   PH_STOP(A, 0);
   // classify: k == |L| -> R (root skipped unless v_s is the earliest vertex of R, Alg 3 L7);
   // later-ordered partial neighbours -> C (Alg 3 L5-6); earlier-ordered ones are never candidates
@@ -1842,7 +1882,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
     const uint32_t j = b + lane;
     const bool occ = j < nocc;
     const uint32_t s = occ ? occl[j] : 0;
-    const uint32_t v = occ ? ldv(keys + s) : 0;
+    const uint32_t v = occ ? (dense ? s : ldv(keys + s)) : 0;
     uint32_t c = 0;
     if (occ) {
       const unsigned long long x = ldv(vals + s);
@@ -1913,7 +1953,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
         if (is2) {
           const uint32_t pos = n2 + __popc(bal & lanemask_lt());
           xrow[pos] = row;
-          xid[pos] = ldv(keys + slot);
+          xid[pos] = dense ? slot : ldv(keys + slot);
         }
         n2 += __popc(bal);
       }
@@ -1977,7 +2017,8 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
       // root node record: candidates in rank order (Alg 2 L6 "smallest first")
       __syncwarp();
       PH_STOP(A, 3);
-      warp_sort_keys(sortbuf, nC, M.sm_sort, (unsigned long long*)rec, 32 - __clz(max(g.n_v, 2u) - 1));
+      if (!dense)  // dense mode: occupied list (and so the candidates) already in rank order
+        warp_sort_keys(sortbuf, nC, M.sm_sort, (unsigned long long*)rec, 32 - __clz(max(g.n_v, 2u) - 1));
       PH_STOP(A, 2);
       uint32_t* ent = rec + kHdr + W4;
       for (uint32_t j = lane; j < nC; j += 32) {
@@ -2019,7 +2060,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
         __syncwarp();
         for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
           if (act && v != r) {
-            const uint32_t h = ht_find(keys, shift, mask, v);
+            const uint32_t h = dense ? v : ht_find(keys, shift, mask, v);
             const unsigned long long x = ldv(vals + h);
             const uint32_t xi = (uint32_t)(x >> 32);
             if (want_cols && xi) atomicOr(cols + (size_t)i * ncw + ((xi - 1) >> 5), 1u << ((xi - 1) & 31));
@@ -2077,7 +2118,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   __syncwarp();
   for (uint32_t j = lane; j < nocc; j += 32) {
     const uint32_t s = occl[j];
-    keys[s] = GMBE_EMPTY;
+    if (!dense) keys[s] = GMBE_EMPTY;
     vals[s] = 0;
   }
   __syncwarp();

@@ -14,7 +14,7 @@ name = sys.argv[1]
 kw = {}
 for a in sys.argv[2:]:
     k, v = a.split("=")
-    kw[k] = int(v)
+    kw[k] = tuple(map(int, v.split("/"))) if k == "part" else int(v)
 nu, nv, e = make_config(name)
 g = gmbe.load(nu, nv, e)
 g.enumerate(**kw)

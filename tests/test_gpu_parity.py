@@ -380,3 +380,32 @@ def test_wide_universe_splitting(gmbe):
                     assert r.bicliques == sorted(o.bicliques), (it, kw)
         finally:
             g.free()
+
+
+def test_dense_mode_roots(gmbe, dense_case):
+    """Dense-mode roots (the warp table indexed by rank, rank-ordered occupied list, no candidate
+    sort) forced on every root (debug 512), alone and with suffix mode (debug 128)."""
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        for dbg in (512, 512 | 128, 512 | 16):
+            r = g.enumerate(records=True, debug=dbg)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques), dbg
+    finally:
+        g.free()
+    rng = np.random.default_rng(78)
+    for it in range(60):
+        nu, nv, e = _rand_graph(rng, nmax=14)
+        o = oracle.oracle_mbe(nu, nv, e, records=True)
+        for dbg in (512, 512 | 128):
+            r = _run(gmbe, nu, nv, e, records=True, debug=dbg)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques)
+    # wide universes (pass 2 builds candidate rows through the dense table)
+    for it in range(6):
+        nu, nv = int(rng.integers(120, 200)), int(rng.integers(20, 40))
+        e = np.argwhere(rng.random((nu, nv)) < 0.35).astype(np.uint32)
+        o = oracle.oracle_mbe(nu, nv, e)
+        for dbg in (512, 512 | 128):
+            _same(_run(gmbe, nu, nv, e, debug=dbg), o)
