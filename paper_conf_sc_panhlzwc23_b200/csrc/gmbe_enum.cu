@@ -1254,7 +1254,7 @@ __device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& 
 struct ThrSmem {
   unsigned long long row[32];  // candidate rows over the universe (the job's top node)
   unsigned long long hv[32];   // hV of each candidate
-  unsigned long long hu[64];   // hU of each universe vertex
+  uint32_t ccol[64];           // bit c: job candidate c is adjacent to universe vertex j
   uint32_t deg[64];            // degree of each universe vertex
   uint32_t id[32];             // rank of each candidate
 };
@@ -1345,8 +1345,8 @@ __device__ bool donate_thr(const Params& P, const TaskCtx& T, uint32_t lmap, Acc
 // smem layout of the column store (the warp's s_sort slice, kSmemSort u64): [0, 128) pattern hash
 // table during setup, then [128, 256) = one ThrCol per universe vertex j
 struct ThrCol {
-  unsigned long long q;  // bit t: Q-pattern t contains j
-  uint32_t c, pad;       // bit c: job candidate c is adjacent to j
+  unsigned long long q;   // bit t: Q-pattern t contains j
+  unsigned long long hu;  // hU of universe vertex j (the emission sum rides on the same loop)
 };
 constexpr uint32_t kThrHash = 128;
 static_assert(kSmemSort * 8 >= kThrHash * 8 + 64 * sizeof(ThrCol), "column store exceeds the s_sort slice");
@@ -1383,8 +1383,6 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     ts->id[lane] = id;
     ts->hv[lane] = P.g.hv[id];
   }
-  ts->hu[lane] = T.hu0;
-  ts->hu[lane + 32] = T.hu1;
   ts->deg[lane] = T.dg0;
   ts->deg[lane + 32] = T.dg1;
   unsigned long long* ht = smem;
@@ -1455,7 +1453,8 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     const uint32_t cj = __ballot_sync(GMBE_FULL, (crow >> j) & 1ull);
     if (lane == (j & 31)) {
       cols[j].q = qj;
-      cols[j].c = cj;
+      cols[j].hu = j < 32 ? T.hu0 : T.hu1;
+      ts->ccol[j] = cj;
     }
   }
   __syncwarp();
@@ -1521,36 +1520,29 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
       const uint32_t donors = __ballot_sync(GMBE_FULL, dmask != 0);
       if (donors) {
         const uint32_t nd = min(__popc(idle), __popc(donors));
-        unsigned long long gL = 0, gSR = 0;
-        uint32_t gC = 0, gRm = 0, gnext = 0, gbd = 0;
-        if (dmask && __popc(donors & lanemask_lt()) < nd) {
+        unsigned long long* slot = smem;  // the setup hash region: 32 slots of 4 words
+        const uint32_t rd = __popc(donors & lanemask_lt());
+        if (dmask && rd < nd) {
           const uint32_t k = __ffs(dmask) - 1;
-          gbd = bd + k;
-          gL = stk[k].L;
-          gSR = stk[k].SR;
-          gC = stk[k].C;
-          gRm = stk[k].Rm;
-          gnext = stk[k].next;
+          unsigned long long* o = slot + 4 * rd;
+          o[0] = stk[k].L;
+          o[1] = stk[k].SR;
+          o[2] = ((unsigned long long)stk[k].Rm << 32) | stk[k].C;
+          o[3] = ((unsigned long long)(bd + k) << 32) | stk[k].next;
           stk[k].next = 32;  // the remaining children of level k are no longer this lane's
           dmask &= ~(1u << k);
         }
+        __syncwarp();
         const uint32_t ir = __popc(idle & lanemask_lt());
-        const bool take = !has && ir < nd;
-        const uint32_t src = take ? __fns(donors, 0, ir + 1) : lane;
-        gL = shfl64(gL, src);
-        gSR = shfl64(gSR, src);
-        gC = __shfl_sync(GMBE_FULL, gC, src);
-        gRm = __shfl_sync(GMBE_FULL, gRm, src);
-        gnext = __shfl_sync(GMBE_FULL, gnext, src);
-        gbd = __shfl_sync(GMBE_FULL, gbd, src);
-        if (take) {
+        if (!has && ir < nd) {
+          const unsigned long long* o = slot + 4 * ir;
           has = true;
-          bd = gbd;
-          L = gL;
-          SR = gSR;
-          C = gC;
-          Rm = gRm;
-          next = gnext;
+          L = o[0];
+          SR = o[1];
+          C = (uint32_t)o[2];
+          Rm = (uint32_t)(o[2] >> 32);
+          next = (uint32_t)o[3];
+          bd = (uint32_t)(o[3] >> 32);
           d = 0;
           dmask = 0;
         }
@@ -1583,29 +1575,37 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     n_nodes++;
     abytes += lc + ksum;
     const uint32_t rl = rlen0 + __popc(Rm) + 1 + __popc(ab);
-    // maximality (Alg 2 L14): |Γ(L')| == |R'|
+    // maximality (Alg 2 L14): |Γ(L')| == |R'|; the emission's SL = Σ_{u∈L'} hU(u) on the same pass
     bool maximal;
+    unsigned long long sl = 0;
     if (lc == 1) {
-      maximal = ts->deg[__ffsll(lp) - 1] == rl;
+      const uint32_t j = __ffsll(lp) - 1;
+      maximal = ts->deg[j] == rl;
+      sl = cols[j].hu;
     } else {  // |L'| >= 2: no Q pattern and no job candidate outside R' may cover L'
       const uint32_t outside = cand_all & ~(Rm | (1u << i) | ab);
-      unsigned long long qa = ~0ull;
+      unsigned long long qa = ~0ull, m = lp;
       uint32_t ca = GMBE_FULL;
-      for (unsigned long long m = lp; m; m &= m - 1) {
-        const ThrCol tc = cols[__ffsll(m) - 1];
+      for (; m; m &= m - 1) {
+        const uint32_t j = __ffsll(m) - 1;
+        const ThrCol tc = cols[j];
         qa &= tc.q;
-        ca &= tc.c;
-        if (!qa && !(ca & outside)) break;
+        sl += tc.hu;
+        ca &= ts->ccol[j];
+        if (!qa && !(ca & outside)) {
+          m &= m - 1;
+          break;
+        }
       }
       maximal = !qa && !(ca & outside);
+      if (maximal)
+        for (; m; m &= m - 1) sl += cols[__ffsll(m) - 1].hu;
     }
     if (!maximal) {
       n_nonmax++;
       continue;
     }
     // Output(L', R') (Alg 2 L15)
-    unsigned long long sl = 0;
-    for (unsigned long long m = lp; m; m &= m - 1) sl += ts->hu[__ffsll(m) - 1];
     const unsigned long long srn = SR + ts->hv[i] + srab;
     const uint32_t rmn = Rm | (1u << i) | ab;
     n_count++;
