@@ -88,8 +88,8 @@ typedef struct {
   uint32_t struct_size;   /* sizeof(gmbe_opts); 0 = treat the struct as all-defaults */
   uint32_t no_prune;      /* 1 disables Thm 4.1 pruning (GMBE-W/O_PRUNE ablation) */
   uint32_t no_split;      /* 1 disables load-aware splitting (Alg 4 L17-26) */
-  uint32_t bound_height;  /* split if min(|L|,|C|) > bound_height ...   (default 8; paper 20) */
-  uint32_t bound_size;    /* ... and min(|L|,|C|)·|C| > bound_size       (default 400; paper 1500,
+  uint32_t bound_height;  /* split if min(|L|,|C|) > bound_height ...   (default 10; paper 20) */
+  uint32_t bound_size;    /* ... and min(|L|,|C|)·|C| > bound_size       (default 500; paper 1500,
                              P:1175; retuned on B200 with scripts/sweep.py) */
   uint32_t warps_per_sm;  /* resident warps per SM of the persistent kernel (0 = auto) */
   uint32_t part_index;    /* root shard: enumerate the roots whose degree rank r satisfies */

@@ -2499,8 +2499,8 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   }
   P.prune = o.no_prune ? 0 : 1;
   P.split = o.no_split ? 0 : 1;
-  P.bound_height = o.bound_height ? o.bound_height : 8;    // paper: 20; retuned for B200
-  P.bound_size = o.bound_size ? o.bound_size : 400;     // paper: 1500; scripts/sweep.py
+  P.bound_height = o.bound_height ? o.bound_height : 10;   // paper: 20; retuned for B200
+  P.bound_size = o.bound_size ? o.bound_size : 500;     // paper: 1500; scripts/sweep.py
   P.hu_side = g.swapped ? 1 : 0;
   P.arena = (uint32_t*)W.arena;
   P.arena_words = arena_words;
