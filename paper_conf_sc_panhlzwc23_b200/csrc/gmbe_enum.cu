@@ -610,31 +610,63 @@ __device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_is_r(const Params& P, const uint
     }
     key = warp_sort32(key);
   } else {
+    // members -> scratch as (deg << 32 | u), lane-parallel over the mask words; u* = the minimum
+    // (no sort: the wide walk below tests 32 members per step in any order)
+    unsigned long long kmin = ~0ull;
     uint32_t c = 0;
-    for (uint32_t w = 0; w < W; w++) {
-      const uint32_t word = lmask[w];
-      const bool b = (word >> lane) & 1u;
-      const uint32_t bal = __ballot_sync(GMBE_FULL, b);
-      if (b) {
-        const uint32_t u = map[w * 32 + lane];
-        scratch[c + __popc(bal & lanemask_lt())] = ((unsigned long long)(g.off_u[u + 1] - g.off_u[u]) << 32) | u;
+    for (uint32_t wb = 0; wb < W; wb += 32) {
+      const uint32_t w = wb + lane;
+      const uint32_t word = w < W ? lmask[w] : 0u;
+      const uint32_t nb = __popc(word);
+      uint32_t inc = nb;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(GMBE_FULL, inc, o);
+        if (lane >= (uint32_t)o) inc += t;
       }
-      c += __popc(bal);
+      uint32_t pos = c + inc - nb;
+      for (uint32_t x = word; x; x &= x - 1) {
+        const uint32_t u = map[w * 32 + __ffs(x) - 1];
+        const unsigned long long kk = ((unsigned long long)(g.off_u[u + 1] - g.off_u[u]) << 32) | u;
+        scratch[pos++] = kk;
+        kmin = min(kmin, kk);
+      }
+      c += __shfl_sync(GMBE_FULL, inc, 31);
     }
+    for (int o = 16; o; o >>= 1) kmin = min(kmin, (unsigned long long)__shfl_xor_sync(GMBE_FULL, kmin, o));
     __syncwarp();
-    warp_sort_keys(scratch, lc, smem);
-    key = lane < lc ? scratch[lane] : ~0ull;
+    key = lane == 0 ? kmin : ~0ull;
   }
   const unsigned long long k0 = __shfl_sync(GMBE_FULL, key, 0);
   const uint32_t d0 = (uint32_t)(k0 >> 32), u0 = (uint32_t)k0;
   if (lc == 1 || d0 <= rlen) return d0 == rlen;  // |Γ(L')| <= deg(u*); |L'| = 1: Γ = N(u*)
-  uint32_t mb = 0, md = 0;  // lane j < 32: (begin, degree) of member j's list
-  if (lane < lc) {
+  uint32_t mb = 0, md = 0;  // lane j < 32: (begin, degree) of member j's list (|L'| <= 32)
+  if (lc <= 32 && lane < lc) {
     mb = g.off_u[(uint32_t)key];
     md = (uint32_t)(key >> 32);
   }
   const uint32_t* n0 = g.adj_u + g.off_u[u0];
   uint32_t count = 0;
+  if (lc > 32) {
+    // wide L': one v ∈ N(u*) at a time, lanes test 32 members per step (a member of Γ(L') -- every
+    // vertex of R' -- costs ⌈|L'|/32⌉ steps instead of |L'| - 1; others usually fail in the first)
+    for (uint32_t b = 0; b < d0; b++) {
+      const uint32_t v = __ldg(n0 + b);
+      bool all = true;
+      for (uint32_t j0 = 0; j0 < lc && all; j0 += 32) {  // (u* itself passes trivially)
+        const uint32_t j = j0 + lane;
+        bool in = true;
+        if (j < lc) {
+          const unsigned long long kj = scratch[j];
+          const uint32_t jb = g.off_u[(uint32_t)kj];
+          in = bsearch_rank(g.adj_u + jb, (uint32_t)(kj >> 32), v);
+        }
+        all = __all_sync(GMBE_FULL, in);
+      }
+      count += all;
+      if (count > rlen) return false;
+    }
+    return count == rlen;
+  }
   for (uint32_t b = 0; b < d0; b += 32) {
     const uint32_t idx = b + lane;
     bool ok = idx < d0;
@@ -789,6 +821,9 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   } else {
     maximal = gamma_is_r(P, lpm, W, T.map, lc, rlen, gscr, smem);
   }
+#ifndef GMBE_PROFILE
+  if ((P.debug & 32) && lane == 0) atomicAdd(&P.ctrl->phase[lc == 1 ? 4 : (T.cols ? 5 : 6)], 1ull);
+#endif
   PH_STOP(A, 5);
   if (!maximal) {
     A.nonmax++;
@@ -797,11 +832,9 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   // Output(L', R') (Alg 2 L15)
   const unsigned long long par_sr = ((unsigned long long)par[7] << 32) | par[6];
   const unsigned long long sr = par_sr + P.g.hv[vid] + warp_sum64(sr_abs);
-  unsigned long long sl = 0;
-  for (uint32_t w = 0; w < W; w++) {
-    const uint32_t word = lpm[w];
-    if ((word >> lane) & 1u) sl += hash_u(P, T.map[w * 32 + lane]);
-  }
+  unsigned long long sl = 0;  // lane t sums the members in words t, t + 32, ...
+  for (uint32_t w = lane; w < W; w += 32)
+    for (uint32_t word = lpm[w]; word; word &= word - 1) sl += hash_u(P, T.map[w * 32 + __ffs(word) - 1]);
   sl = warp_sum64(sl);
   A.count++;
   A.checksum += pair_hash(P, sl, sr);

@@ -21,5 +21,7 @@ for rk in map(int, sys.argv[2:]):
         r = g.enumerate(part=(rk, nroots), phases=True, debug=d)
         r = g.enumerate(part=(rk, nroots), phases=True, debug=d)
         ph = list(r.phase_cycles.values())
-        print("rank %d %s: %.2f ms count %d nodes %d splits %d tasks %d | thr jobs %d nodes %d | reg jobs %d nodes %d" % (
-            rk, extra, r.kernel_ms, r.count, r.nodes, r.splits, r.tasks, ph[0], ph[1], ph[2], ph[3]), flush=True)
+        print("rank %d %s: %.2f ms count %d nodes %d splits %d tasks %d | thr jobs %d nodes %d | reg jobs %d nodes %d"
+              " | wide gamma: deg %d cols %d bsearch %d" % (
+            rk, extra, r.kernel_ms, r.count, r.nodes, r.splits, r.tasks, ph[0], ph[1], ph[2], ph[3], ph[4], ph[5], ph[6]),
+              flush=True)
