@@ -1502,7 +1502,7 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
   uint32_t n_nodes = 0, n_nonmax = 0, n_count = 0;
   unsigned long long abytes = 0, cks = 0;
 #if GMBE_DONATE
-  uint32_t tick = 0;
+  uint32_t tick = 0, hflag = 0;  // hflag: lane 0's in-flight read of ctrl.hungry (consumed 4 steps later)
 #endif
   while (true) {
     if (has) {  // pop (Alg 2 L4) until a node with an untraversed candidate
@@ -1524,7 +1524,12 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     const uint32_t idle = __ballot_sync(GMBE_FULL, !has);
     if (idle == GMBE_FULL) break;
 #if GMBE_DONATE
-    if (P.donate && (++tick & 3) == 0 && hungry(P)) {  // cross-warp donation to idle warps
+    bool want = false;
+    if (P.donate && (++tick & 3) == 0) {
+      want = __shfl_sync(GMBE_FULL, hflag, 0) != 0 || (P.debug & 8);
+      if (lane == 0) hflag = ld_volatile(&P.ctrl->hungry.v) != 0;  // latency hidden until the next check
+    }
+    if (want) {  // cross-warp donation to idle warps
       // the donor: the lane whose shallowest stacked level with untraversed children is the
       // shallowest in the job's tree (the largest piece of remaining work)
       const uint32_t key =
@@ -1827,7 +1832,9 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   uint32_t after = kNone, scanned = wedges;
   if (P.debug & 128) {  // tests: every root in suffix mode
     after = r;
-  } else if (wedges >= GMBE_SUFFIX_MIN && !(P.debug & 64)) {
+  } else if (wedges >= GMBE_SUFFIX_MIN && !(P.debug & 64) &&
+             // a small universe that a dense full scan can afford keeps its Γ index (thread tier)
+             !(l <= 64 && g.n_v <= P.tmax && (uint64_t)g.n_v <= 16ull * wedges && !(P.debug & 256))) {
     uint32_t sp = 0;
     for (uint32_t j = lane; j < l; j += 32) {
       const uint32_t u = Lr[j], ub = g.off_u[u], du = g.off_u[u + 1] - ub;
