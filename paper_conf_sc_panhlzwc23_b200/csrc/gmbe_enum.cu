@@ -1804,6 +1804,12 @@ __device__ bool earlier_dominator(const DevGraph& g, const uint32_t* Lr, uint32_
   }
   return false;
 }
+#ifndef GMBE_DENSE_RATIO
+#define GMBE_DENSE_RATIO 32  // dense root tables when the scanned rank range <= this x the wedges
+#endif
+#ifndef GMBE_SUFFIX_MAX_KEEP_L
+#define GMBE_SUFFIX_MAX_KEEP_L 256  // universes up to this size keep a full (dense) scan and their Γ index
+#endif
 #ifndef GMBE_SUFFIX_MIN
 #define GMBE_SUFFIX_MIN 8192  // roots with at least this many wedges may scan only later ranks
 #endif
@@ -1834,7 +1840,8 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
     after = r;
   } else if (wedges >= GMBE_SUFFIX_MIN && !(P.debug & 64) &&
              // a small universe that a dense full scan can afford keeps its Γ index (thread tier)
-             !(l <= 64 && g.n_v <= P.tmax && (uint64_t)g.n_v <= 16ull * wedges && !(P.debug & 256))) {
+             !(l <= GMBE_SUFFIX_MAX_KEEP_L && g.n_v <= P.tmax && (uint64_t)g.n_v <= 16ull * wedges &&
+               !(P.debug & 256))) {
     uint32_t sp = 0;
     for (uint32_t j = lane; j < l; j += 32) {
       const uint32_t u = Lr[j], ub = g.off_u[u], du = g.off_u[u + 1] - ub;
@@ -1870,7 +1877,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   // a scan of the rank range -- in rank order, so the candidates need no sort.
   const uint32_t lo_v = after != kNone ? r + 1 : 0u;
   const bool dense = !stab && g.n_v <= P.tmax && !(P.debug & 256) &&
-                     ((uint64_t)(g.n_v - lo_v) <= 16ull * scanned || (P.debug & 512));
+                     ((uint64_t)(g.n_v - lo_v) <= (uint64_t)GMBE_DENSE_RATIO * scanned || (P.debug & 512));
   PH_START(A);
   // pass 1 (Alg 3 L2-3)
   uint32_t nocc = 0;
