@@ -1372,6 +1372,12 @@ __device__ bool donate_thr(const Params& P, const TaskCtx& T, uint32_t lmap, Acc
 #ifndef GMBE_SPLIT_WIDE
 #define GMBE_SPLIT_WIDE 32
 #endif
+#ifndef GMBE_DENSE_CS
+#define GMBE_DENSE_CS 0
+#endif
+#ifndef GMBE_THR_DONATE_MASK
+#define GMBE_THR_DONATE_MASK 3  // run_thr checks ctrl.hungry every (mask + 1) steps
+#endif
 #ifndef GMBE_THR_MIN_EST
 #define GMBE_THR_MIN_EST 16  // jobs with fewer adjacency bits (Σ(k-1)) stay on run_reg (setup > work)
 #endif
@@ -1525,7 +1531,7 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     if (idle == GMBE_FULL) break;
 #if GMBE_DONATE
     bool want = false;
-    if (P.donate && (++tick & 3) == 0) {
+    if (P.donate && (++tick & GMBE_THR_DONATE_MASK) == 0) {
       want = __shfl_sync(GMBE_FULL, hflag, 0) != 0 || (P.debug & 8);
       if (lane == 0) hflag = ld_volatile(&P.ctrl->hungry.v) != 0;  // latency hidden until the next check
     }
@@ -1895,7 +1901,11 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
 #pragma unroll
       for (int q = 0; q < 8; q++) {
         const uint32_t v = b + q * 32 + lane;
+#if GMBE_DENSE_CS
+        x[q] = v < g.n_v ? __ldcs(vals + v) : 0ull;  // streaming (evict-first): a one-pass scan
+#else
         x[q] = v < g.n_v ? __ldcg(vals + v) : 0ull;  // L2: pass 1 wrote with atomics
+#endif
       }
 #pragma unroll
       for (int q = 0; q < 8; q++) {

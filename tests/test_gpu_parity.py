@@ -248,7 +248,7 @@ def _gold_cfg():
         return json.load(f)
 
 
-@pytest.mark.parametrize("name", ["yg", "gh", "dblp", "bx", "gh_work"])
+@pytest.mark.parametrize("name", ["yg", "gh", "dblp", "bx", "gh_work", "yg_work", "bx_work"])
 def test_full_config_vs_oracle_golden(gmbe, name):
     gold = _gold_cfg()
     if name not in gold:
