@@ -160,6 +160,9 @@ struct TaskCtx {
 #ifndef GMBE_NI_REG
 #define GMBE_NI_REG 0
 #endif
+#ifndef GMBE_NI_DONATE_THR
+#define GMBE_NI_DONATE_THR 0  // 1: the thread tier's rare paths (cross-warp donation, records) out of line
+#endif
 #ifndef GMBE_NI_GAMMA
 #define GMBE_NI_GAMMA 0
 #endif
@@ -1297,7 +1300,7 @@ struct ThrLevel {
 };
 
 // one output record from one lane: L' = bits of lp over map, R' = the job's R list + candidates rm
-__device__ void write_record_thr(const Params& P, const TaskCtx& T, const ThrSmem* ts, unsigned long long lp,
+__device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) void write_record_thr(const Params& P, const TaskCtx& T, const ThrSmem* ts, unsigned long long lp,
                                  uint32_t nl, uint32_t rlen0, uint32_t rm, uint32_t nr) {
   const unsigned long long need = 2ull + nl + nr;
   const unsigned long long rec = atomicAdd(&P.ctrl->out_rec, 1ull);
@@ -1323,7 +1326,7 @@ __device__ void write_record_thr(const Params& P, const TaskCtx& T, const ThrSme
 
 // Publish lane `src`'s stacked level k (its remaining children) as a subtask for idle warps
 // (cross-warp donation, see donate_reg).  Warp-cooperative; returns whether it was published.
-__device__ bool donate_thr(const Params& P, const TaskCtx& T, uint32_t lmap, Acc& A, const ThrSmem* ts,
+__device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const TaskCtx& T, uint32_t lmap, Acc& A, const ThrSmem* ts,
                            uint32_t nC, uint32_t rlen0, uint32_t src, unsigned long long Lk, unsigned long long SRk,
                            uint32_t Ck, uint32_t Rmk, uint32_t nextk, uint32_t* scratch, const uint32_t* scratch_end) {
   const uint32_t lane = lane_id();
