@@ -159,6 +159,21 @@ typedef struct {
  * Errors: EINVAL (NULL g/out, part_index >= part_count), ENOMEM, ECUDA, EINTERNAL. */
 int gmbe_enumerate(const gmbe_graph* g, const gmbe_opts* opts, gmbe_result* out);
 
+/* Streaming output (the problem statement asks to *enumerate* all maximal
+ * bicliques, Output() of Alg 1/2): every record [|L|, |R|, L ids (caller U ids),
+ * R ids (caller V ids)] is delivered exactly once to `sink`, in batches of whole records
+ * (n_words words holding n_records records, order unspecified), on the calling thread while the
+ * kernel runs.  The kernel writes into a ring of ring_words 32-bit words (rounded up to a power of
+ * two, at least 4x the largest possible record; 0 = 16 Mi words) in mapped pinned host memory and
+ * waits when it is full (back-pressure), so any output size streams through a bounded buffer.
+ * `words` is valid only during the call.  count / checksum / counters are as in gmbe_enumerate;
+ * result.n_written = records delivered (== count).  opts must not carry out_offsets / out_ids.
+ * Errors: as gmbe_enumerate; EINVAL (NULL sink, bounded buffers given, the sink returned non-zero
+ * -- the remaining records are drained but not delivered); EINTERNAL (a producer waited > 20 s). */
+typedef int (*gmbe_sink_fn)(const uint32_t* words, uint64_t n_words, uint64_t n_records, void* user);
+int gmbe_enumerate_stream(const gmbe_graph* g, const gmbe_opts* opts, gmbe_sink_fn sink, void* user,
+                          uint64_t ring_words, gmbe_result* out);
+
 /* gmbe_enumerate keeps its device workspace (node-stack arenas, task slabs, queues) in a
  * per-device pool for reuse by later calls.  This frees the idle workspaces of g's device.
  * NULL-safe. */

@@ -28,7 +28,8 @@ PHASES = ("root_wedges", "classify", "sort", "root_finish", "cand_scan", "maxima
           "lprime", "dequeue")
 EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmbe_node_buf_bound_bytes",
            "gmbe_kernel_launch_count",
-           "gmbe_naive_alloc_bytes", "gmbe_enumerate", "gmbe_release_workspace", "gmbe_last_error")
+           "gmbe_naive_alloc_bytes", "gmbe_enumerate", "gmbe_enumerate_stream", "gmbe_release_workspace",
+           "gmbe_last_error")
 
 _u32, _i32, _u64, _vp = ctypes.c_uint32, ctypes.c_int32, ctypes.c_uint64, ctypes.c_void_p
 
@@ -75,6 +76,9 @@ _lib.gmbe_naive_alloc_bytes.argtypes = [_u64, _u64]
 _lib.gmbe_naive_alloc_bytes.restype = _u64
 _lib.gmbe_enumerate.argtypes = [_vp, ctypes.POINTER(Opts), ctypes.POINTER(CResult)]
 _lib.gmbe_enumerate.restype = ctypes.c_int
+SINK_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.POINTER(ctypes.c_uint32), ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p)
+_lib.gmbe_enumerate_stream.argtypes = [_vp, ctypes.POINTER(Opts), SINK_FN, _vp, _u64, ctypes.POINTER(CResult)]
+_lib.gmbe_enumerate_stream.restype = ctypes.c_int
 _lib.gmbe_kernel_launch_count.argtypes = []
 _lib.gmbe_kernel_launch_count.restype = _u64
 _lib.gmbe_last_error.argtypes = []
@@ -211,6 +215,38 @@ class Graph:
             res.per_root_count = prc[: (self.info()["n_u"] if self.info()["swapped"] else self.info()["n_v"])]
         return res
 
+    def enumerate_stream(self, sink, ring_words=0, prune=True, split=True, bound_height=0, bound_size=0,
+                         part=(0, 1), debug=0, thr_min=0, split_wide=0, stream=None):
+        """gmbe_enumerate_stream: every maximal biclique record is handed to sink(words, n_records)
+        (words: uint32 numpy array of whole records [|L|, |R|, L ids, R ids], valid during the call)
+        while the kernel runs, through a bounded ring in pinned host memory."""
+        o = Opts()
+        o.struct_size = ctypes.sizeof(Opts)
+        o.no_prune = 0 if prune else 1
+        o.no_split = 0 if split else 1
+        o.bound_height, o.bound_size = bound_height, bound_size
+        o.part_index, o.part_count = part
+        o.cuda_stream = _stream_ptr(stream)
+        o.reserved0 = debug
+        o.thr_min, o.split_wide = thr_min, split_wide
+        err = []
+
+        def _cb(words, n_words, n_records, user):
+            try:
+                sink(np.ctypeslib.as_array(words, shape=(int(n_words),)), int(n_records))
+                return 0
+            except Exception as ex:  # reported after the call; the ring is drained
+                err.append(ex)
+                return 1
+
+        cb = SINK_FN(_cb)
+        cr = CResult()
+        rc = _lib.gmbe_enumerate_stream(self._h, ctypes.byref(o), cb, None, ring_words, ctypes.byref(cr))
+        if err:
+            raise err[0]
+        _check(rc)
+        return Result(**{k: getattr(cr, k) for k, _ in CResult._fields_})
+
     def release_workspace(self):
         if self._h:
             _lib.gmbe_release_workspace(self._h)
@@ -238,6 +274,15 @@ def decode_records(offsets, ids):
         out.append((tuple(sorted(ids[o + 2:o + 2 + nl].tolist())),
                     tuple(sorted(ids[o + 2 + nl:o + 2 + nl + nr].tolist()))))
     return sorted(out)
+
+
+def iter_records(words):
+    """Split a batch of streamed records into (L ids, R ids) array pairs (caller roles)."""
+    i, n = 0, len(words)
+    while i < n:
+        nl, nr = int(words[i]), int(words[i + 1])
+        yield words[i + 2:i + 2 + nl], words[i + 2 + nl:i + 2 + nl + nr]
+        i += 2 + nl + nr
 
 
 def load(n_u, n_v, edges, order="degree", device=None, stream=None):

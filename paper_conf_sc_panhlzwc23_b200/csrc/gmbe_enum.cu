@@ -21,6 +21,7 @@
 // counting Γ(L') = ∩_{u∈L'} N(u) over N(u*) for the lowest-degree u* ∈ L' (|Γ(L')| = |R'| iff
 // maximal, since R' ⊆ Γ(L')); for |L'| = 1 this is just deg(u*) == |R'|.
 #include <algorithm>
+#include <atomic>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -50,11 +51,12 @@ struct Ctrl {
   unsigned long long out_rec, out_ids;
   unsigned long long phase[16];
   unsigned int truncated, error;
+  unsigned long long stream_tail;  // streaming output: largest consumer position seen by a producer
 };
 
 static_assert(sizeof(Ctrl) == 1152, "bench.py reports sizeof(Ctrl) as the per-step D2H / H2D control bytes");
 
-enum : unsigned int { kErrArena = 1 };
+enum : unsigned int { kErrArena = 1, kErrStream = 2 };
 
 struct Params {
   DevGraph g;
@@ -78,6 +80,9 @@ struct Params {
   uint64_t out_offsets_cap;
   uint32_t* out_ids;
   uint64_t out_ids_cap;
+  uint32_t* sring;                              // streaming output ring (mapped host memory) or null
+  unsigned long long smask;                     // ring words - 1 (power of two)
+  const unsigned long long* stail;              // host-written consumer position (mapped)
   unsigned long long* per_root;
   unsigned long long* per_root_cycles;
   uint32_t profile;
@@ -532,49 +537,100 @@ __device__ __forceinline__ unsigned long long pair_hash(const Params& P, unsigne
   return P.hu_side ? gmbe_pair_hash(sr, sl) : gmbe_pair_hash(sl, sr);
 }
 
+// ---- output records.  Bounded buffer: record i at out_ids[out_offsets[i]].  Streaming (N2): a ring
+// of words in mapped host memory; a record is [h = 1 + words, words...] at ring positions pos..,
+// published by writing h last (after a system-scope fence); the host consumes in position order,
+// zeroes the words and advances its tail, which producers wait on when the ring is full.
+struct RecOut {
+  uint32_t* p;
+  unsigned long long base, mask;
+  __device__ __forceinline__ uint32_t& at(unsigned long long k) const { return p[(base + k) & mask]; }
+};
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// reserve room for a record of `need` words (one thread); false: nothing to write
+__device__ bool rec_open(const Params& P, unsigned long long need, RecOut& O, unsigned long long& tok) {
+  if (P.sring) {
+    const unsigned long long pos = atomicAdd(&P.ctrl->out_ids, need + 1);
+    atomicAdd(&P.ctrl->out_rec, 1ull);
+    const unsigned long long end = pos + need + 1, cap = P.smask + 1;
+    unsigned long long t0 = 0;
+    while (end - ld_volatile(&P.ctrl->stream_tail) > cap) {  // ring full: back-pressure
+      const unsigned long long t = *(volatile const unsigned long long*)P.stail;  // host memory
+      atomicMax(&P.ctrl->stream_tail, t);
+      if (end - t <= cap) break;
+      const unsigned long long now = globaltimer_ns();
+      if (!t0) t0 = now;
+      if (now - t0 > 20000000000ull) {  // the consumer is gone: give up (the call reports an error)
+        atomicOr(&P.ctrl->error, kErrStream);
+        return false;
+      }
+      __nanosleep(2000);
+    }
+    O = RecOut{P.sring, pos + 1, P.smask};
+    tok = pos;
+    return true;
+  }
+  const unsigned long long rec = atomicAdd(&P.ctrl->out_rec, 1ull);
+  const unsigned long long off = atomicAdd(&P.ctrl->out_ids, need);
+  if (rec >= P.out_offsets_cap || off + need > P.out_ids_cap) {
+    atomicOr(&P.ctrl->truncated, 1u);
+    if (rec < P.out_offsets_cap) P.out_offsets[rec] = ~0ull;
+    return false;
+  }
+  O = RecOut{P.out_ids, off, ~0ull};
+  tok = rec;
+  return true;
+}
+// publish (one thread, after every writer's words are done -- and fenced, when streaming)
+__device__ void rec_close(const Params& P, const RecOut& O, unsigned long long need, unsigned long long tok) {
+  if (P.sring) {
+    __threadfence_system();
+    *(volatile uint32_t*)(P.sring + (tok & P.smask)) = (uint32_t)(need + 1);
+  } else {
+    P.out_offsets[tok] = O.base;
+  }
+}
+
 // Write one output record: L given by bitmap words lmask (W words over map) or, if lmask == null,
 // by the explicit list lids[0..nl); R by ranks rl[0..nr).
 __device__ void write_record(const Params& P, const uint32_t* lmask, uint32_t W, const uint32_t* map,
                              const uint32_t* lids, uint32_t nl, const uint32_t* rl, uint32_t nr) {
   const uint32_t lane = lane_id();
-  unsigned long long rec = 0, off = 0;
   const unsigned long long need = 2ull + nl + nr;
-  if (lane == 0) {
-    rec = atomicAdd(&P.ctrl->out_rec, 1ull);
-    off = atomicAdd(&P.ctrl->out_ids, need);
-  }
-  rec = __shfl_sync(GMBE_FULL, rec, 0);
-  off = __shfl_sync(GMBE_FULL, off, 0);
-  if (rec >= P.out_offsets_cap || off + need > P.out_ids_cap) {
-    if (lane == 0) {
-      atomicOr(&P.ctrl->truncated, 1u);
-      if (rec < P.out_offsets_cap) P.out_offsets[rec] = ~0ull;
-    }
-    return;
-  }
-  uint32_t* o = P.out_ids + off;
+  RecOut O{nullptr, 0, 0};
+  unsigned long long tok = 0;
+  uint32_t ok = 0;
+  if (lane == 0) ok = rec_open(P, need, O, tok);
+  if (!__shfl_sync(GMBE_FULL, ok, 0)) return;
+  O.p = (uint32_t*)__shfl_sync(GMBE_FULL, (unsigned long long)O.p, 0);
+  O.base = __shfl_sync(GMBE_FULL, O.base, 0);
+  O.mask = __shfl_sync(GMBE_FULL, O.mask, 0);
   const bool sw = P.hu_side != 0;  // caller U ids first: the library's L unless swapped
-  uint32_t* lpos = sw ? o + 2 + nr : o + 2;
-  uint32_t* rpos = sw ? o + 2 : o + 2 + nl;
+  const unsigned long long lpos = sw ? 2 + nr : 2, rpos = sw ? 2 : 2 + nl;
   if (lane == 0) {
-    o[0] = sw ? nr : nl;
-    o[1] = sw ? nl : nr;
+    O.at(0) = sw ? nr : nl;
+    O.at(1) = sw ? nl : nr;
   }
-  for (uint32_t j = lane; j < nr; j += 32) rpos[j] = P.g.rank2id[rl[j]];
+  for (uint32_t j = lane; j < nr; j += 32) O.at(rpos + j) = P.g.rank2id[rl[j]];
   if (lmask) {
     uint32_t c = 0;
     for (uint32_t w = 0; w < W; w++) {
       const uint32_t word = lmask[w];
       const bool b = (word >> lane) & 1u;
       const uint32_t bal = __ballot_sync(GMBE_FULL, b);
-      if (b) lpos[c + __popc(bal & lanemask_lt())] = map[w * 32 + lane];
+      if (b) O.at(lpos + c + __popc(bal & lanemask_lt())) = map[w * 32 + lane];
       c += __popc(bal);
     }
   } else {
-    for (uint32_t j = lane; j < nl; j += 32) lpos[j] = lids[j];
+    for (uint32_t j = lane; j < nl; j += 32) O.at(lpos + j) = lids[j];
   }
+  if (P.sring) __threadfence_system();
   __syncwarp();
-  if (lane == 0) P.out_offsets[rec] = off;
+  if (lane == 0) rec_close(P, O, need, tok);
 }
 
 // ---------------------------------------------------------------- maximality (a5)
@@ -845,7 +901,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   if (T.rlist) {
     if (lane == 0) T.rlist[par[5]] = vid;
     __syncwarp();
-    if (P.out_ids) write_record(P, lpm, W, T.map, nullptr, lc, T.rlist, rlen);
+    if (P.out_ids || P.sring) write_record(P, lpm, W, T.map, nullptr, lc, T.rlist, rlen);
   }
   PH_STOP(A, 6);
   if (nCc == 0) return 1;
@@ -1020,7 +1076,7 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
   if (T.rlist) {
     if (lane == 0) T.rlist[par[5]] = vid;
     __syncwarp();
-    if (P.out_ids) write_record(P, ch + kHdr, T.W, T.map, nullptr, lc, T.rlist, rlen);
+    if (P.out_ids || P.sring) write_record(P, ch + kHdr, T.W, T.map, nullptr, lc, T.rlist, rlen);
   }
   PH_STOP(A, 6);
   if (nCc == 0) return 1;
@@ -1221,7 +1277,7 @@ __device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& 
         scratch[1] = (uint32_t)(lp >> 32);
       }
       __syncwarp();
-      if (P.out_ids) write_record(P, scratch, T.W, T.map, nullptr, lc, T.rlist, rl);
+      if (P.out_ids || P.sring) write_record(P, scratch, T.W, T.map, nullptr, lc, T.rlist, rl);
     }
     if (!cd) continue;
     if (split_top && d == 0) {
@@ -1303,25 +1359,19 @@ struct ThrLevel {
 __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) void write_record_thr(const Params& P, const TaskCtx& T, const ThrSmem* ts, unsigned long long lp,
                                  uint32_t nl, uint32_t rlen0, uint32_t rm, uint32_t nr) {
   const unsigned long long need = 2ull + nl + nr;
-  const unsigned long long rec = atomicAdd(&P.ctrl->out_rec, 1ull);
-  const unsigned long long off = atomicAdd(&P.ctrl->out_ids, need);
-  if (rec >= P.out_offsets_cap || off + need > P.out_ids_cap) {
-    atomicOr(&P.ctrl->truncated, 1u);
-    if (rec < P.out_offsets_cap) P.out_offsets[rec] = ~0ull;
-    return;
-  }
-  uint32_t* o = P.out_ids + off;
+  RecOut O;
+  unsigned long long tok;
+  if (!rec_open(P, need, O, tok)) return;
   const bool sw = P.hu_side != 0;
-  uint32_t* lpos = sw ? o + 2 + nr : o + 2;
-  uint32_t* rpos = sw ? o + 2 : o + 2 + nl;
-  o[0] = sw ? nr : nl;
-  o[1] = sw ? nl : nr;
+  const unsigned long long lpos = sw ? 2 + nr : 2, rpos = sw ? 2 : 2 + nl;
+  O.at(0) = sw ? nr : nl;
+  O.at(1) = sw ? nl : nr;
   uint32_t t = 0;
-  for (; t < rlen0; t++) rpos[t] = P.g.rank2id[T.rlist[t]];
-  for (uint32_t m = rm; m; m &= m - 1) rpos[t++] = P.g.rank2id[ts->id[__ffs(m) - 1]];
+  for (; t < rlen0; t++) O.at(rpos + t) = P.g.rank2id[T.rlist[t]];
+  for (uint32_t m = rm; m; m &= m - 1) O.at(rpos + t++) = P.g.rank2id[ts->id[__ffs(m) - 1]];
   t = 0;
-  for (unsigned long long m = lp; m; m &= m - 1) lpos[t++] = T.map[__ffsll(m) - 1];
-  P.out_offsets[rec] = off;
+  for (unsigned long long m = lp; m; m &= m - 1) O.at(lpos + t++) = T.map[__ffsll(m) - 1];
+  rec_close(P, O, need, tok);
 }
 
 // Publish lane `src`'s stacked level k (its remaining children) as a subtask for idle warps
@@ -1658,7 +1708,7 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     n_count++;
     cks += pair_hash(P, sl, srn);
     if (P.per_root) atomicAdd(P.per_root + T.root, 1ull);
-    if (T.rlist && P.out_ids) write_record_thr(P, T, ts, lp, lc, rlen0, rmn, rl);
+    if (T.rlist && (P.out_ids || P.sring)) write_record_thr(P, T, ts, lp, lc, rlen0, rmn, rl);
     if (!cd) continue;
     // push (Alg 2 L16)
     stk[d].L = L;
@@ -1990,7 +2040,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
     if (M.rbuf) {
       if (lane == 0) M.rbuf[0] = r;
       __syncwarp();
-      if (P.out_ids) write_record(P, nullptr, 0, nullptr, Lr, l, M.rbuf, nR + 1);
+      if (P.out_ids || P.sring) write_record(P, nullptr, 0, nullptr, Lr, l, M.rbuf, nR + 1);
     }
     PH_STOP(A, 8);
     if (want_aux && small) {
@@ -2368,6 +2418,10 @@ struct Workspace {
   size_t per_root_cyc_bytes = 0;
   void* shard = nullptr;  // this call's root issue list (part_count > 1) + selection scratch
   size_t shard_bytes = 0;
+  uint32_t* sring_h = nullptr;  // streaming output ring (mapped pinned host memory) + its tail word
+  uint32_t* sring_d = nullptr;
+  uint64_t sring_words = 0;
+  bool sring_dirty = false;
 };
 
 // roots of one shard (rank % part_count == part_index), kept in the graph's issue order
@@ -2426,13 +2480,28 @@ extern "C" void gmbe_release_workspace(const gmbe_graph* G) {
     }
     for (void* p : {w->arena, w->pool, w->rings, w->rbuf, w->ctrl, w->per_root, w->per_root_cyc, w->shard})
       if (p) cudaFree(p);
+    if (w->sring_h) cudaFreeHost(w->sring_h);
     delete w;
     g_ws_idle.erase(g_ws_idle.begin() + i);
   }
   cudaSetDevice(prev);
 }
 
+static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_fn sink, void* user,
+                          uint64_t ring_words, gmbe_result* out);
+
 extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_result* out) {
+  return enumerate_impl(G, opts, nullptr, nullptr, 0, out);
+}
+
+extern "C" int gmbe_enumerate_stream(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_fn sink, void* user,
+                                     uint64_t ring_words, gmbe_result* out) {
+  if (!sink) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate_stream: NULL sink");
+  return enumerate_impl(G, opts, sink, user, ring_words, out);
+}
+
+static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_fn sink, void* user,
+                          uint64_t ring_words, gmbe_result* out) {
   if (!G || !out) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: NULL argument");
   gmbe_opts o{};
   if (opts && opts->struct_size) {
@@ -2443,6 +2512,8 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   if (o.part_index >= parts) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: part_index >= part_count");
   if ((o.out_offsets == nullptr) != (o.out_ids == nullptr))
     return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: out_offsets and out_ids must be given together");
+  if (sink && o.out_ids)
+    return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate_stream: no bounded output buffers with a sink");
   GMBE_CUDA_TRY(cudaSetDevice(G->device));
   cudaStream_t s = o.cuda_stream ? (cudaStream_t)o.cuda_stream : G->stream;
   const DevGraph& g = G->g;
@@ -2519,7 +2590,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   const uint64_t want_cap = o.queue_cap ? o.queue_cap : (1u << 20);
   while (cap < want_cap && cap < (1u << 30)) cap <<= 1;
   if (cap < 16384) cap = 16384;  // > the producers' admission margin
-  const bool want_out = o.out_ids != nullptr;
+  const bool want_out = o.out_ids != nullptr || sink != nullptr;
   const uint32_t rbuf_words = want_out ? (uint32_t)(wb + 64) : 0;
 
   GMBE_CUDA_TRY(ensure(&W.arena, &W.arena_bytes, nwarps * arena_words * 4));
@@ -2578,7 +2649,28 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   P.out_offsets = (unsigned long long*)o.out_offsets;
   P.out_offsets_cap = want_out ? o.out_offsets_cap : 0;
   P.out_ids = o.out_ids;
-  P.out_ids_cap = want_out ? o.out_ids_cap : 0;
+  P.out_ids_cap = o.out_ids ? o.out_ids_cap : 0;
+  if (sink) {
+    // ring of 2^k words >= max(ring_words, 4 * the largest record), mapped pinned host memory
+    uint64_t need = std::max<uint64_t>(ring_words ? ring_words : (1ull << 24),
+                                       4ull * (3ull + g.delta_u + g.delta_v) + 4096);
+    uint64_t words = 1;
+    while (words < need) words <<= 1;
+    if (W.sring_words != words || W.sring_dirty) {
+      if (W.sring_h) cudaFreeHost(W.sring_h);
+      W.sring_h = nullptr;
+      W.sring_words = 0;
+      GMBE_CUDA_TRY(cudaHostAlloc((void**)&W.sring_h, (words + 32) * 4, cudaHostAllocMapped));
+      std::memset(W.sring_h, 0, (words + 32) * 4);
+      GMBE_CUDA_TRY(cudaHostGetDevicePointer((void**)&W.sring_d, W.sring_h, 0));
+      W.sring_words = words;
+      W.sring_dirty = false;
+    }
+    *(volatile unsigned long long*)(W.sring_h + words + 16) = 0;  // consumer tail
+    P.sring = W.sring_d;
+    P.smask = words - 1;
+    P.stail = (const unsigned long long*)(W.sring_d + words + 16);
+  }
   P.per_root = o.per_root_count ? (unsigned long long*)W.per_root : nullptr;
   P.per_root_cycles = o.per_root_cycles ? (unsigned long long*)W.per_root_cyc : nullptr;
   P.profile = o.phase_cycles ? 1 : 0;
@@ -2604,6 +2696,65 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   const cudaError_t le = cudaGetLastError();
   GMBE_CUDA_TRY(cudaEventRecord(e1, s));
   GMBE_CUDA_TRY(le);
+  uint64_t streamed = 0;
+  int sink_rc = 0;
+  if (sink) {
+    // consumer (this thread, while the kernel runs): deliver records in ring order, zero their
+    // words, then advance the tail the producers wait on
+    volatile uint32_t* R = W.sring_h;
+    volatile unsigned long long* tail = (volatile unsigned long long*)(W.sring_h + W.sring_words + 16);
+    const uint64_t mask = W.sring_words - 1;
+    std::vector<uint32_t> batch;
+    uint64_t c = 0, nb = 0, final_pos = ~0ull;
+    bool done = false, failed = false;
+    auto flush = [&]() {
+      if (!batch.empty()) {
+        if (!sink_rc) sink_rc = sink(batch.data(), batch.size(), nb, user);
+        batch.clear();
+        nb = 0;
+      }
+    };
+    while (true) {
+      const uint32_t h = R[c & mask];
+      if (h) {
+        std::atomic_thread_fence(std::memory_order_acquire);  // the words were published before h
+        uint32_t* base = W.sring_h;
+        const uint64_t first = (c + 1) & mask, n = h - 1, n1 = std::min<uint64_t>(n, W.sring_words - first);
+        const size_t old = batch.size();
+        batch.resize(old + n);
+        std::memcpy(batch.data() + old, base + first, n1 * 4);
+        std::memset(base + first, 0, n1 * 4);
+        if (n1 < n) {
+          std::memcpy(batch.data() + old + n1, base, (n - n1) * 4);
+          std::memset(base, 0, (n - n1) * 4);
+        }
+        R[c & mask] = 0;
+        c += h;
+        nb++;
+        streamed++;
+        std::atomic_thread_fence(std::memory_order_seq_cst);
+        *tail = c;
+        if (batch.size() >= (1u << 20)) flush();
+        continue;
+      }
+      flush();
+      if (done) {
+        if (c >= final_pos || failed) break;
+        continue;  // the last records' words are still arriving over the bus
+      }
+      const cudaError_t q = cudaEventQuery(e1);
+      if (q == cudaSuccess) {
+        Ctrl hc2{};
+        GMBE_CUDA_TRY(cudaMemcpy(&hc2, W.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost));
+        final_pos = hc2.out_ids;
+        failed = hc2.error != 0;
+        done = true;
+      } else if (q != cudaErrorNotReady) {
+        GMBE_CUDA_TRY(q);
+      }
+    }
+    if (failed || c != final_pos) W.sring_dirty = true;
+  }
   GMBE_CUDA_TRY(cudaMemcpyAsync(&hc, W.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s));
   GMBE_CUDA_TRY(cudaStreamSynchronize(s));
   float ms = 0;
@@ -2625,7 +2776,7 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   }
   out->count = hc.count;
   out->checksum = hc.checksum;
-  out->n_written = hc.out_rec < P.out_offsets_cap ? hc.out_rec : P.out_offsets_cap;
+  out->n_written = sink ? streamed : (hc.out_rec < P.out_offsets_cap ? hc.out_rec : P.out_offsets_cap);
   out->truncated = hc.truncated;
   out->roots_run = hc.roots_run;
   out->nodes = hc.nodes;
@@ -2637,10 +2788,15 @@ extern "C" int gmbe_enumerate(const gmbe_graph* G, const gmbe_opts* opts, gmbe_r
   out->kernel_ms = ms;
   if (o.phase_cycles)
     for (int k = 0; k < 16; k++) o.phase_cycles[k] = hc.phase[k];
+  if (hc.error & kErrStream) {
+    W.clean = false;
+    return gmbe_set_error(GMBE_EINTERNAL, "gmbe_enumerate_stream: the consumer stopped draining the ring");
+  }
   if (hc.error) {
     W.clean = false;
     return gmbe_set_error(GMBE_EINTERNAL,
                           "gmbe_enumerate: per-warp workspace exceeded; raise opts.arena_words");
   }
+  if (sink_rc) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate_stream: the sink returned non-zero");
   return GMBE_OK;
 }

@@ -409,3 +409,72 @@ def test_dense_mode_roots(gmbe, dense_case):
         o = oracle.oracle_mbe(nu, nv, e)
         for dbg in (512, 512 | 128):
             _same(_run(gmbe, nu, nv, e, debug=dbg), o)
+
+
+# ---------------------------------------------------------------- streaming output (N2)
+def _stream_all(g, **kw):
+    got = []
+
+    def sink(words, n_records):
+        got.extend((tuple(sorted(l.tolist())), tuple(sorted(r.tolist()))) for l, r in gmbe_mod().iter_records(words))
+    r = g.enumerate_stream(sink, **kw)
+    return r, got
+
+
+def gmbe_mod():
+    import paper_conf_sc_panhlzwc23_b200 as m
+    return m
+
+
+def test_stream_sets_small_ring(gmbe, dense_case):
+    """Every record streamed exactly once through a ring far smaller than the output (wrap-around
+    and back-pressure), on every tier: sets equal the oracle's, count == records delivered."""
+    from oracle.brute import checksum
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        for kw in (dict(), dict(debug=16), dict(debug=8), dict(debug=128 | 512), dict(thr_min=1)):
+            r, got = _stream_all(g, ring_words=1, **kw)  # rounded up to the minimum ring
+            assert (r.count, r.checksum) == (o.count, o.checksum), kw
+            assert r.n_written == r.count == len(got), kw
+            assert sorted(got) == sorted(o.bicliques), kw
+            assert checksum(got) == o.checksum
+    finally:
+        g.free()
+    for n in (8, 12):  # crown graphs: 2^n - 2 records
+        nu, nv, e = crown_edges(n)
+        g = gmbe.load(nu, nv, e)
+        try:
+            r, got = _stream_all(g, ring_words=1)
+            assert r.count == len(got) == 2 ** n - 2 and len(set(got)) == len(got)
+            assert checksum(got) == r.checksum
+        finally:
+            g.free()
+
+
+def test_stream_full_config(gmbe):
+    """A full-size config streamed with the default ring: delivered records reproduce the golden
+    count and checksum (computed on the host from the streamed sets)."""
+    from oracle.brute import checksum
+    gd = _gold_cfg()["gh"]
+    nu, nv, e = make_config("gh")
+    g = gmbe.load(nu, nv, e)
+    try:
+        r, got = _stream_all(g)
+        assert (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16))
+        assert r.n_written == len(got) == gd["count"]
+        assert checksum(got) == int(gd["checksum"], 16)
+    finally:
+        g.free()
+
+
+def test_stream_rejects_bounded_buffers(gmbe):
+    nu, nv, e = g0_edges()
+    g = gmbe.load(nu, nv, e)
+    try:
+        with pytest.raises(ZeroDivisionError):  # a sink error propagates after the ring is drained
+            g.enumerate_stream(lambda w, n: 1 / 0)
+        r, got = _stream_all(g)  # the workspace stays usable
+        assert r.count == 6 and len(got) == 6
+    finally:
+        g.free()
