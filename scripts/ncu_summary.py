@@ -23,8 +23,20 @@ keys = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__thread_inst_executed_per_inst_executed.ratio", "sm__warps_active.avg.pct_of_peak_sustained_active",
         "smsp__issue_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
         "launch__grid_size", "launch__block_size", "l1tex__t_sector_hit_rate.pct", "lts__t_sector_hit_rate.pct",
-        "dram__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum"]
+        "dram__throughput.avg.pct_of_peak_sustained_elapsed", "smsp__inst_executed.sum",
+        "lts__t_sectors.sum", "lts__throughput.avg.pct_of_peak_sustained_elapsed",
+        "l1tex__throughput.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed"]
 summ = {k: m[k][0] + " " + m[k][1] for k in keys if k in m}
+try:  # derived: achieved L2 and DRAM bandwidth, warp execution efficiency
+    t_s = float(m["gpu__time_duration.sum"][0].replace(",", "")) * {"ms": 1e-3, "us": 1e-6, "s": 1.0}[m["gpu__time_duration.sum"][1].strip()]
+    l2 = float(m["lts__t_sectors.sum"][0].replace(",", "")) * 32
+    summ["derived_l2_GBps"] = round(l2 / t_s / 1e9, 1)
+    mult = {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1.0}
+    dr = sum(float(m[k][0].replace(",", "")) * mult[m[k][1].strip()] for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
+    summ["derived_dram_GBps"] = round(dr / t_s / 1e9, 1)
+    summ["derived_warp_execution_efficiency"] = round(float(m["smsp__thread_inst_executed_per_inst_executed.ratio"][0]) / 32, 3)
+except (KeyError, ValueError):
+    pass
 st = {h[len("smsp__pcsamp_warps_issue_stalled_"):]: float(v.replace(",", "") or 0) for h, (v, u) in m.items()
       if h.startswith("smsp__pcsamp_warps_issue_stalled_") and not h.endswith("not_issued")}
 tot = sum(st.values()) or 1
