@@ -2266,12 +2266,16 @@ __device__ __forceinline__ unsigned long long tl_info(unsigned long long nodes, 
 #ifndef GMBE_MIN_BLOCKS
 #define GMBE_MIN_BLOCKS 3  // 80 registers: 24 resident warps per SM (measured best on gh_work)
 #endif
-__global__ void __launch_bounds__(256, GMBE_MIN_BLOCKS) k_enum(const Params P) {
-  __shared__ unsigned long long s_sort[8][kSmemSort];
-  __shared__ unsigned long long s_tvals[8][kSmemTable ? kSmemTable : 1];
-  __shared__ uint32_t s_tkeys[8][kSmemTable ? kSmemTable : 1];
-  __shared__ uint32_t s_tocc[8][kSmemTable ? kSmemTable / 2 : 1];
-  __shared__ ThrSmem s_thr[8];
+#ifndef GMBE_WPB
+#define GMBE_WPB 8  // warps per block
+#endif
+constexpr uint32_t kWpb = GMBE_WPB;
+__global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const Params P) {
+  __shared__ unsigned long long s_sort[kWpb][kSmemSort];
+  __shared__ unsigned long long s_tvals[kWpb][kSmemTable ? kSmemTable : 1];
+  __shared__ uint32_t s_tkeys[kWpb][kSmemTable ? kSmemTable : 1];
+  __shared__ uint32_t s_tocc[kWpb][kSmemTable ? kSmemTable / 2 : 1];
+  __shared__ ThrSmem s_thr[kWpb];
   const uint32_t lane = lane_id();
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   uint32_t* base = P.arena + (uint64_t)gw * P.arena_words;
@@ -2527,16 +2531,16 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
 
   if (W.sms == 0) {  // per-device constants, queried once per workspace
     GMBE_CUDA_TRY(cudaDeviceGetAttribute(&W.sms, cudaDevAttrMultiProcessorCount, G->device));
-    GMBE_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&W.bps_max, k_enum, 256, 0));
+    GMBE_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&W.bps_max, k_enum, 32 * kWpb, 0));
   }
-  uint32_t wps = o.warps_per_sm ? o.warps_per_sm : 32;
-  if (wps < 8) wps = 8;
+  uint32_t wps = o.warps_per_sm ? o.warps_per_sm : 64;
+  if (wps < kWpb) wps = kWpb;
   if (wps > 64) wps = 64;
-  uint32_t bps = wps / 8;
+  uint32_t bps = wps / kWpb;
   if ((int)bps > W.bps_max) bps = W.bps_max;
   if (bps < 1) bps = 1;
   const uint32_t blocks = (uint32_t)W.sms * bps;
-  const uint64_t nwarps = (uint64_t)blocks * 8;
+  const uint64_t nwarps = (uint64_t)blocks * kWpb;
 
   // per-warp arena: clean hash table sized for the largest root's wedges, its occupied list, and
   // the dynamic region (root record, node stack, Γ index), bounded by free memory.  A cached layout
@@ -2692,7 +2696,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   GMBE_CUDA_TRY(cudaEventCreate(&e0));
   GMBE_CUDA_TRY(cudaEventCreate(&e1));
   GMBE_CUDA_TRY(cudaEventRecord(e0, s));
-  if (P.n_roots > 0) k_enum<<<blocks, 256, 0, s>>>(P), gmbe_note_launch();
+  if (P.n_roots > 0) k_enum<<<blocks, 32 * kWpb, 0, s>>>(P), gmbe_note_launch();
   const cudaError_t le = cudaGetLastError();
   GMBE_CUDA_TRY(cudaEventRecord(e1, s));
   GMBE_CUDA_TRY(le);
