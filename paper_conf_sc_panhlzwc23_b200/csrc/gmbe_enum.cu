@@ -945,8 +945,8 @@ __device__ void small_task_init(const Params& P, TaskCtx& T, uint32_t lmap) {
       if (lane + 32 < T.nx) T.xr1 = xrow[lane + 32];
     }
     const uint32_t* coff = T.gx + 4 + 2 * T.gx[0] + r4(T.gx[0]);
-    const uint32_t l = T.gx[1];
-    T.gxl = coff + r4(l + 1);
+    const uint32_t l = T.nx > 64 ? T.gx[1] : 0u;  // |X2| <= 64: no lists (rows are lane-resident)
+    T.gxl = coff + r4(T.gx[1] + 1);
     if (lane < l) {
       T.go0 = coff[lane];
       T.gl0 = coff[lane + 1] - T.go0;
@@ -1883,6 +1883,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   const uint32_t lb = g.off_v[r], l = g.off_v[r + 1] - lb;
   if (l == 0) return false;  // isolated vertex: in no biclique (A17)
   const uint32_t* Lr = g.adj_v + lb;
+  const unsigned long long hv_r = g.hv[r];  // issued early, consumed at the root's emission
   uint32_t wp = 0;
   for (uint32_t j = lane; j < l; j += 32) {
     const uint32_t u = Lr[j];
@@ -2030,10 +2031,10 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   const uint64_t rec_need = kHdr + W4 + (uint64_t)nC * E;
   if (sort_fits && !skip && fits(P, rec + rec_need + 64, M.dyn_end)) {
     A.roots_run++;
-    sr = warp_sum64(sr) + g.hv[r];
+    sr = warp_sum64r(sr) + hv_r;
     unsigned long long sl = 0;
     for (uint32_t j = lane; j < l; j += 32) sl += hash_u(P, Lr[j]);
-    sl = warp_sum64(sl);
+    sl = warp_sum64r(sl);
     A.count++;  // emit (L_r, R_r) (A5)
     A.checksum += pair_hash(P, sl, sr);
     if (P.per_root && lane == 0) atomicAdd(P.per_root + r, 1ull);
@@ -2086,7 +2087,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
         }
       }
       uint32_t carry = 0, cur0 = 0, cur1 = 0;
-      for (uint32_t h = 0; h < 2; h++) {
+      for (uint32_t h = 0; h < 2 && nx2 > 64; h++) {  // (|X2| <= 64: rows lane-resident, no lists)
         const uint32_t j = h * 32 + lane;
         const uint32_t c = h ? cnt1 : cnt0;
         uint32_t inc = c;
@@ -2100,7 +2101,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
         else cur1 = ex;
         carry += __shfl_sync(GMBE_FULL, inc, 31);
       }
-      if (lane == 0 && l == 64) coff[64] = carry;
+      if (lane == 0 && l == 64 && nx2 > 64) coff[64] = carry;
       __syncwarp();
       for (uint32_t b = 0; b < nx2 && nx2 > 64; b += 32) {
         const uint32_t x = b + lane;
