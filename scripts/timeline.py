@@ -39,5 +39,9 @@ out = dict(config=name, kernel_ms=r.kernel_ms, records=len(t), span_us=float(end
                          start_us=round(float(t0[i]), 1), dur_us=round(float(dur[i]), 1),
                          nodes=int(t[i, 3] >> 32), l_top=int((t[i, 3] >> 16) & 0xFFFF), c_top=int(t[i, 3] & 0xFFFF))
                     for i in order],
-           last_end_by_kind={int(k): round(float(t1[kind == k].max()), 1) for k in np.unique(kind)})
+           last_end_by_kind={int(k): round(float(t1[kind == k].max()), 1) for k in np.unique(kind)},
+           last_to_end=[dict(kind=int(kind[i]), root=int(t[i, 0] & 0xFFFFFFFFFFFF), start_us=round(float(t0[i]), 1),
+                             dur_us=round(float(dur[i]), 1), nodes=int(t[i, 3] >> 32),
+                             l_top=int((t[i, 3] >> 16) & 0xFFFF), c_top=int(t[i, 3] & 0xFFFF))
+                        for i in np.argsort(-t1)[:8]])
 print(json.dumps(out))
