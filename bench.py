@@ -35,6 +35,8 @@ def _args():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
+    ap.add_argument("--static", action="store_true",
+                    help="N>1: fixed degree-rank interleave instead of the shared root cursor (N1)")
     return ap.parse_args()
 
 
@@ -185,26 +187,40 @@ def main():
     e_dev = torch.from_numpy(e.astype(np.int32)).to(dev)                   # resident in HBM
     e_host = torch.from_numpy(e.astype(np.int32)).pin_memory()             # for the e2e leg
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)          # > 126 MB L2
+    # N > 1: every rank draws roots from one shared cursor in rank 0's HBM, unless
+    # --static or the cursor cannot be mapped (then the degree-rank interleave)
+    dr = None
+    if ws > 1:
+        dr = gdist.DynamicRoots(rank, ws, local, dev=dev) if not a.static else None
+        if dr is not None and not dr.dynamic:
+            dr = None
     part = (rank, ws)
 
     host_ms = {"load": [], "enumerate": []}
+    abytes_cand = []
 
     def step(edges, kernel_ms):
         t0 = time.perf_counter()
         g = gmbe.load(nu, nv, edges, device=local, stream=stream)
         t1 = time.perf_counter()
-        r = g.enumerate(part=part, stream=stream)
+        if dr is not None:
+            r, tot = dr.enumerate(g, stream=stream)
+        else:
+            r = g.enumerate(part=part, stream=stream)
         t2 = time.perf_counter()
         g.free()
         host_ms["load"].append(1e3 * (t1 - t0))
         host_ms["enumerate"].append(1e3 * (t2 - t1))
         kernel_ms.append(r.kernel_ms)
+        abytes_cand.append(r.algo_bytes_cand)
+        if dr is not None:
+            return tot
         # the only cross-GPU exchange: one NCCL all-reduce of the int64-viewed totals (N > 1)
         return gdist.allreduce_result(r, device=dev)
 
-    # canonical work of this shard (identical in every schedule; reported by every run)
+    # canonical work of this shard (static parts: identical in every schedule)
     g = gmbe.load(nu, nv, e_dev, device=local, stream=stream)
-    rc = g.enumerate(part=part, stream=stream)
+    rc = dr.enumerate(g, stream=stream)[0] if dr is not None else g.enumerate(part=part, stream=stream)
     g.free()
 
     kms = []
@@ -238,9 +254,12 @@ def main():
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         g = gmbe.load(nu, nv, e_host.numpy(), device=local, stream=stream)
-        r = g.enumerate(part=part, stream=stream)
+        if dr is not None:
+            total_e2e = dr.enumerate(g, stream=stream)[1]["count"]
+        else:
+            r = g.enumerate(part=part, stream=stream)
+            total_e2e = gdist.allreduce_result(r, device=dev)["count"]
         g.free()
-        total_e2e = gdist.allreduce_result(r, device=dev)["count"]
         e1.record(stream)
         e1.synchronize()
         e2e_ms.append(e0.elapsed_time(e1))
@@ -248,9 +267,15 @@ def main():
     t_rank = sum(dev_ms) / len(dev_ms)
     t_e2e = sum(e2e_ms) / len(e2e_ms)
     k_rank = sum(kms) / len(kms)
+    ab_rank = sum(abytes_cand[-a.steps:]) / a.steps  # this rank's candidate bytes per timed launch
     tt = torch.tensor([t_rank, t_e2e], dtype=torch.float64, device=dev)
+    rank_ms = [k_rank]
     if ws > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        kk = torch.tensor([k_rank], dtype=torch.float64, device=dev)
+        ga = [torch.zeros_like(kk) for _ in range(ws)]
+        dist.all_gather(ga, kk)
+        rank_ms = [float(x) for x in ga]
     t_step, t_e2e = float(tt[0]), float(tt[1])
     count = res["count"]
     checksum = res["checksum"]
@@ -265,13 +290,20 @@ def main():
         # algorithmic bytes of this launch (SURVEY 8(d) definition, oracle-counted on the canonical
         # tree): the golden total, apportioned to this shard by its exactly-counted candidate bytes
         if gold and gold.get("algo_bytes") and gold.get("algo_bytes_cand"):
-            abytes = gold["algo_bytes"] * (rc.algo_bytes_cand / gold["algo_bytes_cand"])
+            abytes = gold["algo_bytes"] * (ab_rank / gold["algo_bytes_cand"])
             adef = "SURVEY 8(d) (oracle golden, filtered-Q)"
         else:
-            abytes = rc.algo_bytes_cand
+            abytes = ab_rank
             adef = "wedge + candidate terms only (no golden)"
         achieved = abytes / (k_rank * 1e-3) / 1e9 if k_rank > 0 else 0.0
         st = graph_stats(nu, nv, e)
+        if ws == 1:
+            par = "single GPU (one persistent kernel, device root cursor)"
+        elif dr is not None:
+            par = ("shared root cursor x%d (rank 0 HBM via CUDA IPC, system-scope atomics over NVLink)"
+                   " + NCCL all-reduce" % ws)
+        else:
+            par = "root-shard x%d (degree-rank interleave) + NCCL all-reduce" % ws
         line = {
             "metric": METRIC, "value": count / (t_step * 1e-3), "unit": "bicliques/s",
             "n_gpus": ws, "steps": a.steps, "warmup": a.warmup, "ms_per_step": t_step,
@@ -280,10 +312,12 @@ def main():
             "config": {"workload": a.config, "n_u": nu, "n_v": nv, "m": st["m"],
                        "delta_u": st["delta_u"], "delta_v": st["delta_v"], "seed": 0,
                        "bicliques": count, "checksum": hex(checksum), "oracle_parity": parity,
-                       "parallelism": "root-shard x%d (degree-rank interleave) + NCCL all-reduce" % ws,
+                       "parallelism": par,
                        "l2": "flushed between steps (256 MiB memset)",
                        "step": "device CSR build + enumerate (+ all-reduce)"},
             "kernel_ms": k_rank,
+            "rank_kernel_ms": rank_ms,
+            "imbalance": max(rank_ms) / (sum(rank_ms) / len(rank_ms)) if rank_ms and sum(rank_ms) > 0 else 1.0,
             "host_wall_ms": {k: round(sum(v[-a.steps:]) / max(1, len(v[-a.steps:])), 3) for k, v in host_ms.items()},
             "e2e": {"value": count / (t_e2e * 1e-3), "unit": "bicliques/s",
                     "h2d_bytes_per_step": int(m * 8) + CTRL_BYTES, "d2h_bytes_per_step": CTRL_BYTES},
@@ -292,7 +326,7 @@ def main():
                          "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": _traffic(a.config),
                          "algo_bytes_per_launch": abytes, "algo_bytes_definition": adef,
-                         "algo_bytes_cand": rc.algo_bytes_cand},
+                         "algo_bytes_cand": ab_rank},
             "work": {"nodes": rc.nodes, "nonmax": rc.nonmax, "roots_run": rc.roots_run,
                      "splits": rc.splits, "tasks": rc.tasks, "donations": rc.donations},
             "clocks": clocks,
@@ -304,7 +338,11 @@ def main():
                                     "sample": "%s (%d bicliques, %.1f s)" % (sample, c, dt)}
         print(json.dumps(line), flush=True)
     if ws > 1:
+        if dr is not None and rank != 0:
+            dr.close()  # importers unmap first, then the owner frees
         dist.barrier()
+        if dr is not None and rank == 0:
+            dr.close()
         dist.destroy_process_group()
 
 

@@ -136,6 +136,16 @@ typedef struct {
   uint32_t thr_min;       /* thread-level tier: jobs (<= 32 candidates over <= 64 universe bits)
                              with Σ_c (|N(c) ∩ L| - 1) >= thr_min run one subtree per lane
                              (default 16; UINT32_MAX disables the tier) */
+  /* Dynamic cross-GPU root distribution (Sec 5: GPUs take
+   * root tasks from one shared pool instead of a fixed split).  NULL = off.  Otherwise a
+   * device-accessible uint64 counter shared by several concurrent gmbe_enumerate calls on replicas
+   * of the SAME graph (same edges, same order; possibly on other GPUs or in other processes, see
+   * gmbe_shared_cursor_*): every call draws positions of the graph's full root issue list from it
+   * with system-scope atomics, so the union of the calls enumerates every root exactly once and
+   * their counts / checksums add (mod 2^64) to the single-call result.  Requires part_count <= 1.
+   * The counter must be 0 when the first call starts and must not be reused (or reset) before every
+   * call sharing it has returned. */
+  uint64_t* root_cursor;
 } gmbe_opts;
 
 typedef struct {
@@ -173,6 +183,26 @@ int gmbe_enumerate(const gmbe_graph* g, const gmbe_opts* opts, gmbe_result* out)
 typedef int (*gmbe_sink_fn)(const uint32_t* words, uint64_t n_words, uint64_t n_records, void* user);
 int gmbe_enumerate_stream(const gmbe_graph* g, const gmbe_opts* opts, gmbe_sink_fn sink, void* user,
                           uint64_t ring_words, gmbe_result* out);
+
+/* Shared root cursors for gmbe_opts.root_cursor.  A cursor block holds
+ * GMBE_CURSOR_SLOTS independent uint64 counters in device memory of one GPU (the owner); other
+ * processes map it through CUDA IPC (peer access over NVLink / NVSwitch is enabled on open, or the
+ * same device in another process).  Rotating slots lets consecutive calls run with a single
+ * synchronisation between them: call k uses slot k % SLOTS and the owner zeroes slot (k+1) % SLOTS
+ * before call k starts.
+ *   Slot i is the counter at dptr + 16·i (one 128-byte line each).
+ *   create : cudaMalloc on `device` (zeroed, synchronous); *dptr = device pointer of slot 0;
+ *            ipc_handle (GMBE_IPC_HANDLE_BYTES bytes, may be NULL) receives the export handle.
+ *   open   : map another process's block on `device` (the current GPU of this process);
+ *            *dptr = this process's pointer to slot 0.  EINVAL for NULL args, ECUDA if CUDA IPC or
+ *            peer access is unavailable (the caller falls back to static parts).
+ *   reset  : zero slot `slot` of the block at dptr, stream-ordered on `cuda_stream` (NULL = legacy).
+ *   close  : unmap (opened) or free (created, owner = 1) the block.  NULL-safe. */
+enum { GMBE_CURSOR_SLOTS = 16, GMBE_IPC_HANDLE_BYTES = 64 };
+int gmbe_shared_cursor_create(int32_t device, uint64_t** dptr, void* ipc_handle);
+int gmbe_shared_cursor_open(const void* ipc_handle, int32_t device, uint64_t** dptr);
+int gmbe_shared_cursor_reset(uint64_t* dptr, uint32_t slot, void* cuda_stream);
+void gmbe_shared_cursor_close(uint64_t* dptr, int32_t owner);
 
 /* gmbe_enumerate keeps its device workspace (node-stack arenas, task slabs, queues) in a
  * per-device pool for reuse by later calls.  This frees the idle workspaces of g's device.

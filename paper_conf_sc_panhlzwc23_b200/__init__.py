@@ -29,7 +29,9 @@ PHASES = ("root_wedges", "classify", "sort", "root_finish", "cand_scan", "maxima
 EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmbe_node_buf_bound_bytes",
            "gmbe_kernel_launch_count",
            "gmbe_naive_alloc_bytes", "gmbe_enumerate", "gmbe_enumerate_stream", "gmbe_release_workspace",
-           "gmbe_last_error")
+           "gmbe_last_error", "gmbe_shared_cursor_create", "gmbe_shared_cursor_open",
+           "gmbe_shared_cursor_reset", "gmbe_shared_cursor_close")
+CURSOR_SLOTS, IPC_HANDLE_BYTES = 16, 64
 
 _u32, _i32, _u64, _vp = ctypes.c_uint32, ctypes.c_int32, ctypes.c_uint64, ctypes.c_void_p
 
@@ -53,7 +55,7 @@ class Opts(ctypes.Structure):
                 ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("phase_cycles", _vp), ("timeline", _vp), ("timeline_cap", _u64),
                 ("arena_words", _u64),
                 ("pool_words", _u64), ("queue_cap", _u64), ("cuda_stream", _vp),
-                ("split_wide", _u32), ("thr_min", _u32)]
+                ("split_wide", _u32), ("thr_min", _u32), ("root_cursor", _vp)]
 
 
 class CResult(ctypes.Structure):
@@ -74,6 +76,14 @@ _lib.gmbe_node_buf_bound_bytes.argtypes = [_u64, _u64]
 _lib.gmbe_node_buf_bound_bytes.restype = _u64
 _lib.gmbe_naive_alloc_bytes.argtypes = [_u64, _u64]
 _lib.gmbe_naive_alloc_bytes.restype = _u64
+_lib.gmbe_shared_cursor_create.argtypes = [_i32, ctypes.POINTER(_vp), _vp]
+_lib.gmbe_shared_cursor_create.restype = ctypes.c_int
+_lib.gmbe_shared_cursor_open.argtypes = [_vp, _i32, ctypes.POINTER(_vp)]
+_lib.gmbe_shared_cursor_open.restype = ctypes.c_int
+_lib.gmbe_shared_cursor_reset.argtypes = [_vp, _u32, _vp]
+_lib.gmbe_shared_cursor_reset.restype = ctypes.c_int
+_lib.gmbe_shared_cursor_close.argtypes = [_vp, _i32]
+_lib.gmbe_shared_cursor_close.restype = None
 _lib.gmbe_enumerate.argtypes = [_vp, ctypes.POINTER(Opts), ctypes.POINTER(CResult)]
 _lib.gmbe_enumerate.restype = ctypes.c_int
 SINK_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.POINTER(ctypes.c_uint32), ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p)
@@ -155,8 +165,10 @@ class Graph:
 
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
-                  per_root=False, root_cycles=False, phases=False, timeline=0, debug=0, thr_min=0, split_wide=0, arena_words=0, pool_words=0, queue_cap=0, stream=None):
-        """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them."""
+                  per_root=False, root_cycles=False, phases=False, timeline=0, debug=0, thr_min=0, split_wide=0, arena_words=0, pool_words=0, queue_cap=0, stream=None,
+                  root_cursor=None):
+        """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them.
+        root_cursor: device address (int) of a shared root-cursor slot (SharedCursor.slot_ptr)."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
         o.no_prune = 0 if prune else 1
@@ -167,6 +179,7 @@ class Graph:
         o.cuda_stream = _stream_ptr(stream)
         o.reserved0 = debug
         o.thr_min, o.split_wide = thr_min, split_wide
+        o.root_cursor = root_cursor
         bufs = None
         if records:
             import torch
@@ -261,6 +274,44 @@ class Graph:
             self.free()
         except Exception:
             pass
+
+
+class SharedCursor:
+    """A block of CURSOR_SLOTS root cursors in one GPU's memory, shareable across processes through
+    CUDA IPC (gmbe_shared_cursor_*).  create() on the owner, handle() -> bytes to
+    broadcast, open(handle) on the others."""
+
+    def __init__(self, ptr, owner):
+        self.ptr, self.owner = ptr, owner
+
+    @classmethod
+    def create(cls, device):
+        p, h = _vp(), ctypes.create_string_buffer(IPC_HANDLE_BYTES)
+        _check(_lib.gmbe_shared_cursor_create(device, ctypes.byref(p), h))
+        c = cls(p.value, 1)
+        c._handle = h.raw
+        return c
+
+    @classmethod
+    def open(cls, handle, device):
+        p = _vp()
+        buf = ctypes.create_string_buffer(bytes(handle), IPC_HANDLE_BYTES)
+        _check(_lib.gmbe_shared_cursor_open(buf, device, ctypes.byref(p)))
+        return cls(p.value, 0)
+
+    def handle(self):
+        return self._handle
+
+    def slot_ptr(self, k):
+        return self.ptr + 128 * (k % CURSOR_SLOTS)
+
+    def reset(self, k, stream=None):
+        _check(_lib.gmbe_shared_cursor_reset(self.ptr, k % CURSOR_SLOTS, _stream_ptr(stream)))
+
+    def close(self):
+        if self.ptr:
+            _lib.gmbe_shared_cursor_close(self.ptr, self.owner)
+            self.ptr = None
 
 
 def decode_records(offsets, ids):

@@ -95,6 +95,7 @@ struct Params {
   uint32_t split_wide;   // wide-universe split threshold on |C|·⌈|L|/32⌉ (opts.split_wide)
   unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1, info]*
   uint64_t timeline_cap;
+  unsigned long long* shared_cursor;  // N1: root cursor shared across GPUs / processes (opts.root_cursor)
 };
 
 struct Acc {
@@ -2344,7 +2345,8 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
       unsigned long long t = 0;
       if (lane == 0) {
         atomicAdd(&P.ctrl->pending.v, 1ull);
-        t = atomicAdd(&P.ctrl->root_cursor.v, 1ull);
+        // N1: a cursor shared by every GPU takes a system-scope atomic over NVLink
+        t = P.shared_cursor ? atomicAdd_system(P.shared_cursor, 1ull) : atomicAdd(&P.ctrl->root_cursor.v, 1ull);
       }
       t = __shfl_sync(GMBE_FULL, t, 0);
       if (t < P.n_roots) {
@@ -2515,6 +2517,8 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   }
   const uint32_t parts = o.part_count ? o.part_count : 1;
   if (o.part_index >= parts) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: part_index >= part_count");
+  if (o.root_cursor && parts > 1)
+    return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: root_cursor needs part_count <= 1");
   if ((o.out_offsets == nullptr) != (o.out_ids == nullptr))
     return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: out_offsets and out_ids must be given together");
   if (sink && o.out_ids)
@@ -2685,6 +2689,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   P.split_wide = o.split_wide ? o.split_wide : GMBE_SPLIT_WIDE;
   P.timeline = (unsigned long long*)o.timeline;
   P.timeline_cap = o.timeline_cap;
+  P.shared_cursor = (unsigned long long*)o.root_cursor;
   if (P.timeline) GMBE_CUDA_TRY(cudaMemsetAsync(P.timeline, 0, 8, s));
 
   Ctrl hc{};
@@ -2804,4 +2809,55 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   }
   if (sink_rc) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate_stream: the sink returned non-zero");
   return GMBE_OK;
+}
+
+// ---- shared root cursors -------------------------------------------------------
+static_assert(sizeof(cudaIpcMemHandle_t) <= GMBE_IPC_HANDLE_BYTES, "IPC handle size");
+
+extern "C" int gmbe_shared_cursor_create(int32_t device, uint64_t** dptr, void* ipc_handle) {
+  if (!dptr) return gmbe_set_error(GMBE_EINVAL, "gmbe_shared_cursor_create: NULL dptr");
+  *dptr = nullptr;
+  GMBE_CUDA_TRY(cudaSetDevice(device));
+  void* p = nullptr;
+  GMBE_CUDA_TRY(cudaMalloc(&p, GMBE_CURSOR_SLOTS * 128));
+  cudaError_t e = cudaMemset(p, 0, GMBE_CURSOR_SLOTS * 128);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess && ipc_handle) {
+    cudaIpcMemHandle_t h;
+    e = cudaIpcGetMemHandle(&h, p);
+    if (e == cudaSuccess) {
+      std::memset(ipc_handle, 0, GMBE_IPC_HANDLE_BYTES);
+      std::memcpy(ipc_handle, &h, sizeof(h));
+    }
+  }
+  if (e != cudaSuccess) {
+    cudaFree(p);
+    return gmbe_set_error(GMBE_ECUDA, std::string("gmbe_shared_cursor_create: ") + cudaGetErrorString(e));
+  }
+  *dptr = (uint64_t*)p;
+  return GMBE_OK;
+}
+
+extern "C" int gmbe_shared_cursor_open(const void* ipc_handle, int32_t device, uint64_t** dptr) {
+  if (!dptr || !ipc_handle) return gmbe_set_error(GMBE_EINVAL, "gmbe_shared_cursor_open: NULL argument");
+  *dptr = nullptr;
+  GMBE_CUDA_TRY(cudaSetDevice(device));
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, ipc_handle, sizeof(h));
+  void* p = nullptr;
+  GMBE_CUDA_TRY(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
+  *dptr = (uint64_t*)p;
+  return GMBE_OK;
+}
+
+extern "C" int gmbe_shared_cursor_reset(uint64_t* dptr, uint32_t slot, void* cuda_stream) {
+  if (!dptr || slot >= GMBE_CURSOR_SLOTS) return gmbe_set_error(GMBE_EINVAL, "gmbe_shared_cursor_reset: bad argument");
+  GMBE_CUDA_TRY(cudaMemsetAsync(dptr + 16 * slot, 0, 8, (cudaStream_t)cuda_stream));
+  return GMBE_OK;
+}
+
+extern "C" void gmbe_shared_cursor_close(uint64_t* dptr, int32_t owner) {
+  if (!dptr) return;
+  if (owner) cudaFree(dptr);
+  else cudaIpcCloseMemHandle(dptr);
 }

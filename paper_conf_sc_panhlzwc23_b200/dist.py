@@ -7,6 +7,14 @@ rank gets the same mix of light and heavy roots), with no exchange during the se
 collective is one all-reduce (SUM) of the per-rank [count, checksum, ...] vector -- NCCL over NVLink /
 NVSwitch on the B200 box, gloo in the CPU tests.  uint64 sums travel as int64 views: two's-complement
 addition is bit-identical mod 2^64, so the reduced checksum equals the single-GPU one exactly.
+
+DynamicRoots (the paper's GPUs draw root tasks from one shared pool):
+instead of the fixed interleave, every rank draws positions of the (identical, replicated) root
+issue list from ONE counter in rank 0's HBM, mapped into the other processes through CUDA IPC and
+advanced with system-scope atomics over NVLink / NVSwitch.  Heavy roots are issued first, so the
+ranks finish together whatever the degree tail.  The per-call all-reduce doubles as the one
+synchronisation the rotating cursor slots need (gmbe.h, gmbe_shared_cursor_*).  If any rank cannot
+map the cursor, every rank falls back to the static interleave (agreed by one MIN all-reduce).
 """
 import torch
 import torch.distributed as dist
@@ -50,3 +58,64 @@ def enumerate_sharded(graph, rank, world, group=None, device="cpu", **kw):
     """Enumerate this rank's root shard of `graph` and all-reduce the totals."""
     r = graph.enumerate(part=shard_of(rank, world), **kw)
     return r, allreduce_result(r, group=group, device=device)
+
+
+class DynamicRoots:
+    """Per-process handle of the shared root cursor (N1).  Collective constructor: every rank of
+    `group` must build it, in the same order.  `device`: this rank's CUDA device index; `dev`:
+    the torch device of the NCCL tensors (cpu for gloo)."""
+
+    def __init__(self, rank, world, device, group=None, dev="cpu", cursor_factory=None):
+        self.rank, self.world, self.group, self.dev = rank, world, group, dev
+        self.k = 0
+        self.cursor = None
+        if cursor_factory is None:
+            from paper_conf_sc_panhlzwc23_b200 import SharedCursor
+            cursor_factory = SharedCursor
+        err = None
+        box = [None]
+        if rank == 0:
+            try:
+                self.cursor = cursor_factory.create(device)
+                box[0] = self.cursor.handle()
+            except Exception as ex:  # no CUDA IPC here: everyone falls back
+                err = ex
+        if world > 1:
+            dist.broadcast_object_list(box, src=0, group=group)
+            if rank != 0 and box[0] is not None:
+                try:
+                    self.cursor = cursor_factory.open(box[0], device)
+                except Exception as ex:
+                    err = ex
+            ok = torch.tensor([0 if self.cursor is None else 1], dtype=torch.int64, device=dev)
+            dist.all_reduce(ok, op=dist.ReduceOp.MIN, group=group)
+            agreed = bool(ok.item())
+        else:
+            agreed = self.cursor is not None
+        if not agreed:
+            if self.cursor is not None:
+                self.cursor.close()
+            self.cursor = None
+        self.error = None if agreed else str(err or "a peer rank could not map the cursor")
+
+    @property
+    def dynamic(self):
+        return self.cursor is not None
+
+    def enumerate(self, graph, stream=None, **kw):
+        """One collective call: enumerate this rank's share of the roots and all-reduce the totals.
+        Returns (this rank's Result, the reduced dict)."""
+        k = self.k
+        self.k += 1
+        if self.cursor is None:
+            r = graph.enumerate(part=shard_of(self.rank, self.world), stream=stream, **kw)
+        else:
+            if self.rank == 0:  # slot k+1 is zero before any rank can reach call k+1
+                self.cursor.reset(k + 1, stream=stream)
+            r = graph.enumerate(root_cursor=self.cursor.slot_ptr(k), stream=stream, **kw)
+        return r, allreduce_result(r, group=self.group, device=self.dev)
+
+    def close(self):
+        if self.cursor is not None:
+            self.cursor.close()
+            self.cursor = None

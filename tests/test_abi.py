@@ -38,14 +38,15 @@ def test_exports_every_declared_symbol(gmbe):
 def test_struct_layouts_match_c(gmbe, tmp_path):
     c = tmp_path / "sz.c"
     c.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "gmbe.h"\nint main(){'
-                 'printf("%zu %zu %zu %zu %zu %zu\\n", sizeof(gmbe_load_opts), sizeof(gmbe_graph_info),'
+                 'printf("%zu %zu %zu %zu %zu %zu %zu\\n", sizeof(gmbe_load_opts), sizeof(gmbe_graph_info),'
                  ' sizeof(gmbe_opts), sizeof(gmbe_result), offsetof(gmbe_opts, out_offsets),'
-                 ' offsetof(gmbe_result, kernel_ms));return 0;}')
+                 ' offsetof(gmbe_result, kernel_ms), offsetof(gmbe_opts, root_cursor));return 0;}')
     exe = tmp_path / "sz"
     subprocess.check_call(["gcc", "-I", os.path.dirname(HDR), str(c), "-o", str(exe)])
     got = list(map(int, subprocess.check_output([str(exe)]).split()))
     want = [ctypes.sizeof(gmbe.LoadOpts), ctypes.sizeof(gmbe.GraphInfo), ctypes.sizeof(gmbe.Opts),
-            ctypes.sizeof(gmbe.CResult), gmbe.Opts.out_offsets.offset, gmbe.CResult.kernel_ms.offset]
+            ctypes.sizeof(gmbe.CResult), gmbe.Opts.out_offsets.offset, gmbe.CResult.kernel_ms.offset,
+            gmbe.Opts.root_cursor.offset]
     assert got == want
 
 

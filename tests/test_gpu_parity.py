@@ -478,3 +478,99 @@ def test_stream_rejects_bounded_buffers(gmbe):
         assert r.count == 6 and len(got) == 6
     finally:
         g.free()
+
+
+# ---------------------------------------------------------------- N1: shared root cursor
+def test_shared_cursor_concurrent_calls(gmbe):
+    """Two concurrent gmbe_enumerate calls (two replicas, two streams, two host threads) draw roots
+    from one shared cursor with system-scope atomics: their results add up to the whole-graph golden
+    bit-exactly, whoever wins which root.  An exhausted slot yields nothing; a reset slot everything."""
+    import threading
+    import torch
+    gd = _gold_cfg()["gh"]
+    nu, nv, e = make_config("gh")
+    cur = gmbe.SharedCursor.create(0)
+    gs = [gmbe.load(nu, nv, e) for _ in range(2)]
+    ss = [torch.cuda.Stream() for _ in range(2)]
+    try:
+        for k in range(3):
+            out = [None, None]
+
+            def run(i):
+                out[i] = gs[i].enumerate(root_cursor=cur.slot_ptr(k), stream=ss[i])
+
+            th = [threading.Thread(target=run, args=(i,)) for i in range(2)]
+            for t in th:
+                t.start()
+            for t in th:
+                t.join()
+            assert sum(r.count for r in out) == gd["count"]
+            assert sum(r.checksum for r in out) % (1 << 64) == int(gd["checksum"], 16)
+            assert sum(r.nodes for r in out) == gd["nodes"]
+            assert sum(r.roots_run for r in out) == gd["roots_run"]
+        r = gs[0].enumerate(root_cursor=cur.slot_ptr(0))  # slot 0 is exhausted
+        assert r.count == 0 and r.roots_run == 0
+        cur.reset(0)
+        torch.cuda.synchronize()
+        r = gs[0].enumerate(root_cursor=cur.slot_ptr(0))
+        assert (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16))
+        with pytest.raises(gmbe.GmbeError):
+            gs[0].enumerate(root_cursor=cur.slot_ptr(1), part=(0, 2))
+    finally:
+        for g in gs:
+            g.free()
+        cur.close()
+
+
+def _ipc_worker(rank, world, port, name, q):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_panhlzwc23_b200 as m
+    from paper_conf_sc_panhlzwc23_b200 import dist as gdist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        dr = gdist.DynamicRoots(rank, world, device=0)
+        nu, nv, e = make_config(name)
+        g = m.load(nu, nv, e)
+        outs = []
+        for _ in range(3):
+            r, tot = dr.enumerate(g)
+            outs.append((r.count, tot["count"], tot["checksum"], tot["nodes"]))
+        q.put((rank, dr.dynamic, dr.error, outs))
+        g.free()
+        if rank:
+            dr.close()
+        dist.barrier()
+        if not rank:
+            dr.close()
+    finally:
+        dist.destroy_process_group()
+
+
+def test_dynamic_roots_two_processes_ipc(gmbe):
+    """bench.py's N>1 launch shape with the N1 cursor: two processes (here both on GPU 0), rank 0's
+    cursor mapped into rank 1 through CUDA IPC; three consecutive collective calls."""
+    import socket
+    import torch.multiprocessing as mp
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    gd = _gold_cfg()["gh"]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_ipc_worker, args=(r, 2, port, "gh", q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    out = sorted(q.get(timeout=600) for _ in range(2))
+    for p in ps:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    for rank, dyn, err, outs in out:
+        assert dyn, err
+        for mine, cnt, cks, nodes in outs:
+            assert (cnt, cks, nodes) == (gd["count"], int(gd["checksum"], 16), gd["nodes"])
+    for step in range(3):
+        assert sum(o[3][step][0] for o in out) == gd["count"]
