@@ -35,8 +35,10 @@ def _args():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
-    ap.add_argument("--static", action="store_true",
-                    help="N>1: fixed degree-rank interleave instead of the shared root cursor (N1)")
+    ap.add_argument("--partition", default="dynamic", choices=["dynamic", "interleave", "cost"],
+                    help="N>1 root distribution: shared root cursor (N1), degree-rank interleave "
+                         "(SURVEY 8(e)) or cost-model snake/LPT parts (N4)")
+    ap.add_argument("--static", action="store_true", help="alias of --partition interleave")
     return ap.parse_args()
 
 
@@ -191,9 +193,12 @@ def main():
     # --static or the cursor cannot be mapped (then the degree-rank interleave)
     dr = None
     if ws > 1:
-        dr = gdist.DynamicRoots(rank, ws, local, dev=dev) if not a.static else None
+        if a.static:
+            a.partition = "interleave"
+        dr = gdist.DynamicRoots(rank, ws, local, dev=dev) if a.partition == "dynamic" else None
         if dr is not None and not dr.dynamic:
             dr = None
+    pmode = a.partition if a.partition in ("interleave", "cost") else "interleave"
     part = (rank, ws)
 
     host_ms = {"load": [], "enumerate": []}
@@ -206,7 +211,7 @@ def main():
         if dr is not None:
             r, tot = dr.enumerate(g, stream=stream)
         else:
-            r = g.enumerate(part=part, stream=stream)
+            r = g.enumerate(part=part, stream=stream, part_mode=pmode)
         t2 = time.perf_counter()
         g.free()
         host_ms["load"].append(1e3 * (t1 - t0))
@@ -220,7 +225,8 @@ def main():
 
     # canonical work of this shard (static parts: identical in every schedule)
     g = gmbe.load(nu, nv, e_dev, device=local, stream=stream)
-    rc = dr.enumerate(g, stream=stream)[0] if dr is not None else g.enumerate(part=part, stream=stream)
+    rc = (dr.enumerate(g, stream=stream)[0] if dr is not None
+          else g.enumerate(part=part, stream=stream, part_mode=pmode))
     g.free()
 
     kms = []
@@ -257,7 +263,7 @@ def main():
         if dr is not None:
             total_e2e = dr.enumerate(g, stream=stream)[1]["count"]
         else:
-            r = g.enumerate(part=part, stream=stream)
+            r = g.enumerate(part=part, stream=stream, part_mode=pmode)
             total_e2e = gdist.allreduce_result(r, device=dev)["count"]
         g.free()
         e1.record(stream)
@@ -302,6 +308,8 @@ def main():
         elif dr is not None:
             par = ("shared root cursor x%d (rank 0 HBM via CUDA IPC, system-scope atomics over NVLink)"
                    " + NCCL all-reduce" % ws)
+        elif pmode == "cost":
+            par = "root-shard x%d (cost-model snake/LPT on wedge counts) + NCCL all-reduce" % ws
         else:
             par = "root-shard x%d (degree-rank interleave) + NCCL all-reduce" % ws
         line = {

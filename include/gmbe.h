@@ -146,7 +146,18 @@ typedef struct {
    * The counter must be 0 when the first call starts and must not be reused (or reset) before every
    * call sharing it has returned. */
   uint64_t* root_cursor;
+  /* How part_index / part_count split the roots:
+   *   GMBE_PART_INTERLEAVE (0): degree rank r % part_count == part_index;
+   *   GMBE_PART_COST (1): cost-model LPT -- the roots in the issue order (root cost = its Alg 3
+   *     wedge count Σ_{u∈N(v_s)} |N(u)|, heaviest first) dealt out in snake order (block b of
+   *     part_count consecutive roots goes to parts 0..P-1 if b is even, P-1..0 if odd), the
+   *     parallel form of greedy LPT on a sorted cost list.  Either way the parts partition the
+   *     roots, so counts / checksums add (mod 2^64). */
+  uint32_t part_mode;
+  uint32_t reserved2;     /* must be 0 */
 } gmbe_opts;
+
+enum { GMBE_PART_INTERLEAVE = 0, GMBE_PART_COST = 1 };
 
 typedef struct {
   uint64_t count;         /* maximal bicliques enumerated (this shard) */

@@ -32,6 +32,7 @@ EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmb
            "gmbe_last_error", "gmbe_shared_cursor_create", "gmbe_shared_cursor_open",
            "gmbe_shared_cursor_reset", "gmbe_shared_cursor_close")
 CURSOR_SLOTS, IPC_HANDLE_BYTES = 16, 64
+PART_MODE = {"interleave": 0, "cost": 1}
 
 _u32, _i32, _u64, _vp = ctypes.c_uint32, ctypes.c_int32, ctypes.c_uint64, ctypes.c_void_p
 
@@ -55,7 +56,8 @@ class Opts(ctypes.Structure):
                 ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("phase_cycles", _vp), ("timeline", _vp), ("timeline_cap", _u64),
                 ("arena_words", _u64),
                 ("pool_words", _u64), ("queue_cap", _u64), ("cuda_stream", _vp),
-                ("split_wide", _u32), ("thr_min", _u32), ("root_cursor", _vp)]
+                ("split_wide", _u32), ("thr_min", _u32), ("root_cursor", _vp),
+                ("part_mode", _u32), ("reserved2", _u32)]
 
 
 class CResult(ctypes.Structure):
@@ -166,9 +168,10 @@ class Graph:
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
                   per_root=False, root_cycles=False, phases=False, timeline=0, debug=0, thr_min=0, split_wide=0, arena_words=0, pool_words=0, queue_cap=0, stream=None,
-                  root_cursor=None):
+                  root_cursor=None, part_mode="interleave"):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them.
-        root_cursor: device address (int) of a shared root-cursor slot (SharedCursor.slot_ptr)."""
+        root_cursor: device address (int) of a shared root-cursor slot (SharedCursor.slot_ptr).
+        part_mode: how `part` splits the roots -- "interleave" (degree rank mod N) or "cost" (N4)."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
         o.no_prune = 0 if prune else 1
@@ -180,6 +183,7 @@ class Graph:
         o.reserved0 = debug
         o.thr_min, o.split_wide = thr_min, split_wide
         o.root_cursor = root_cursor
+        o.part_mode = PART_MODE[part_mode]
         bufs = None
         if records:
             import torch

@@ -2437,6 +2437,24 @@ struct ShardOf {
   __host__ __device__ __forceinline__ bool operator()(const uint32_t& r) const { return r % pc == pi; }
 };
 
+// N4 cost-model parts: position p = b·pc + j of the issue list (heaviest wedge count first) goes to
+// part j in even blocks b and to part pc-1-j in odd ones (snake deal = parallel greedy LPT)
+__global__ void k_snake_part(const uint32_t* __restrict__ issue, uint32_t n, uint32_t pc, uint32_t pi,
+                             uint32_t* __restrict__ out) {
+  const uint32_t nb = (n + pc - 1) / pc;
+  for (uint32_t b = blockIdx.x * blockDim.x + threadIdx.x; b < nb; b += gridDim.x * blockDim.x) {
+    const uint64_t p = (uint64_t)b * pc + ((b & 1) ? pc - 1 - pi : pi);
+    if (p < n) out[b] = issue[p];
+  }
+}
+
+static uint32_t snake_count(uint32_t n, uint32_t pc, uint32_t pi) {
+  const uint32_t full = n / pc, rem = n % pc;  // blocks 0..full-1 are complete
+  if (!rem) return full;
+  const uint32_t j = (full & 1) ? pc - 1 - pi : pi;  // the partial block b = full
+  return full + (j < rem ? 1 : 0);
+}
+
 cudaError_t ensure(void** p, size_t* have, size_t need) {
   if (*have >= need && *p) return cudaSuccess;
   if (*p) cudaFree(*p);
@@ -2517,6 +2535,8 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   }
   const uint32_t parts = o.part_count ? o.part_count : 1;
   if (o.part_index >= parts) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: part_index >= part_count");
+  if (o.part_mode > GMBE_PART_COST || o.reserved2)
+    return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: bad part_mode / reserved2");
   if (o.root_cursor && parts > 1)
     return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: root_cursor needs part_count <= 1");
   if ((o.out_offsets == nullptr) != (o.out_ids == nullptr))
@@ -2626,7 +2646,15 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   P.part_count = parts;
   P.n_roots = g.n_v > o.part_index ? (g.n_v - o.part_index + parts - 1) / parts : 0;
   P.issue = g.issue;
-  if (parts > 1 && P.n_roots) {
+  if (parts > 1 && o.part_mode == GMBE_PART_COST) {
+    P.n_roots = snake_count(g.n_v, parts, o.part_index);
+    if (P.n_roots) {
+      GMBE_CUDA_TRY(ensure(&W.shard, &W.shard_bytes, (size_t)P.n_roots * 4));
+      k_snake_part<<<(P.n_roots + 255) / 256, 256, 0, s>>>(g.issue, g.n_v, parts, o.part_index, (uint32_t*)W.shard);
+      gmbe_note_launch();
+      P.issue = (const uint32_t*)W.shard;
+    }
+  } else if (parts > 1 && P.n_roots) {
     size_t tb = 0;
     GMBE_CUDA_TRY(cub::DeviceSelect::If(nullptr, tb, g.issue, (uint32_t*)nullptr, (int*)nullptr, (int)g.n_v,
                                         ShardOf{parts, o.part_index}, s));

@@ -65,8 +65,10 @@ class DynamicRoots:
     `group` must build it, in the same order.  `device`: this rank's CUDA device index; `dev`:
     the torch device of the NCCL tensors (cpu for gloo)."""
 
-    def __init__(self, rank, world, device, group=None, dev="cpu", cursor_factory=None):
+    def __init__(self, rank, world, device, group=None, dev="cpu", cursor_factory=None,
+                 fallback="interleave"):
         self.rank, self.world, self.group, self.dev = rank, world, group, dev
+        self.fallback = fallback  # part_mode of the static split if the cursor is unavailable
         self.k = 0
         self.cursor = None
         if cursor_factory is None:
@@ -108,6 +110,8 @@ class DynamicRoots:
         k = self.k
         self.k += 1
         if self.cursor is None:
+            if self.fallback != "interleave":
+                kw["part_mode"] = self.fallback
             r = graph.enumerate(part=shard_of(self.rank, self.world), stream=stream, **kw)
         else:
             if self.rank == 0:  # slot k+1 is zero before any rank can reach call k+1

@@ -1,5 +1,5 @@
 """Projected multi-GPU balance: time each root shard part=(i, N) of a config on one GPU.
-    python scripts/shard_times.py gh_work 2 4 8"""
+    python scripts/shard_times.py gh_work 2 4 8 [mode=cost]"""
 import json
 import os
 import sys
@@ -10,17 +10,18 @@ from gmbe_inputs import make_config  # noqa: E402
 
 name = sys.argv[1]
 kw = dict(a.split("=") for a in sys.argv[2:] if "=" in a)
+mode = kw.pop("mode", "interleave")
 kw = {k: int(v) for k, v in kw.items()}
 nu, nv, e = make_config(name)
 g = gmbe.load(nu, nv, e)
 full = g.enumerate(**kw)
 full = g.enumerate(**kw)
-out = {"config": name, "opts": kw, "n1_ms": full.kernel_ms, "count": full.count}
+out = {"config": name, "mode": mode, "opts": kw, "n1_ms": full.kernel_ms, "count": full.count}
 for n in [int(a) for a in sys.argv[2:] if "=" not in a]:
     ts, cnt = [], 0
     for i in range(n):
-        g.enumerate(part=(i, n), **kw)
-        r = g.enumerate(part=(i, n), **kw)
+        g.enumerate(part=(i, n), part_mode=mode, **kw)
+        r = g.enumerate(part=(i, n), part_mode=mode, **kw)
         ts.append(r.kernel_ms)
         cnt += r.count
     assert cnt == full.count
