@@ -178,10 +178,19 @@ def main():
 
     ws, rank, local = _dist()
     assert ws == a.gpus or ws == 1, "launch with torchrun --nproc-per-node %d" % a.gpus
+    # GMBE_BENCH_SHARE_GPU=1 (tests only): every rank on GPU 0 over gloo, to exercise the N>1 code
+    # path (shared cursor through CUDA IPC, collectives, the JSON line) on a one-GPU box; its numbers
+    # are not multi-GPU measurements and the line says so
+    share = os.environ.get("GMBE_BENCH_SHARE_GPU") == "1"
+    if share:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream(dev)
 
     nu, nv, e = make_config(a.config)
@@ -278,10 +287,10 @@ def main():
     rank_ms = [k_rank]
     if ws > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        kk = torch.tensor([k_rank], dtype=torch.float64, device=dev)
-        ga = [torch.zeros_like(kk) for _ in range(ws)]
-        dist.all_gather(ga, kk)
-        rank_ms = [float(x) for x in ga]
+        kk = torch.zeros(ws, dtype=torch.float64, device=dev)  # per-rank kernel ms (gather by SUM)
+        kk[rank] = k_rank
+        dist.all_reduce(kk, op=dist.ReduceOp.SUM)
+        rank_ms = [float(x) for x in kk.cpu()]
     t_step, t_e2e = float(tt[0]), float(tt[1])
     count = res["count"]
     checksum = res["checksum"]
@@ -312,6 +321,8 @@ def main():
             par = "root-shard x%d (cost-model snake/LPT on wedge counts) + NCCL all-reduce" % ws
         else:
             par = "root-shard x%d (degree-rank interleave) + NCCL all-reduce" % ws
+        if share and ws > 1:
+            par += " [TEST: all ranks share GPU 0 over gloo; not a multi-GPU measurement]"
         line = {
             "metric": METRIC, "value": count / (t_step * 1e-3), "unit": "bicliques/s",
             "n_gpus": ws, "steps": a.steps, "warmup": a.warmup, "ms_per_step": t_step,
