@@ -200,6 +200,14 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)          # > 126 MB L2
     # N > 1: every rank draws roots from one shared cursor in rank 0's HBM, unless
     # --static or the cursor cannot be mapped (then the degree-rank interleave)
+    if share and ws > 1:
+        # ranks sharing one GPU size their (free-memory-capped) workspaces one after the other
+        for i in range(ws):
+            if rank == i:
+                g = gmbe.load(nu, nv, e_dev, device=local, stream=stream)
+                g.enumerate(part=(rank, ws), stream=stream)
+                g.free()
+            dist.barrier()
     dr = None
     if ws > 1:
         if a.static:

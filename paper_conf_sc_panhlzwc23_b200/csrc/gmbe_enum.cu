@@ -297,6 +297,9 @@ __device__ __forceinline__ uint32_t upper_rank(const uint32_t* a, uint32_t n, ui
 // Visit every wedge (i, v): u_i = L[i], v ∈ N(u_i), load-balanced across the warp.
 // f(i, v, active) is called by all 32 lanes each step.  after != kNone: only the wedges to ranks
 // > after (a suffix of each rank-sorted list).
+#ifndef GMBE_WEDGE_UNROLL
+#define GMBE_WEDGE_UNROLL 1
+#endif
 template <class F>
 __device__ __forceinline__ void for_each_wedge(const DevGraph& g, const uint32_t* L, uint32_t l, F f,
                                                uint32_t after = 0xffffffffu) {
@@ -321,20 +324,30 @@ __device__ __forceinline__ void for_each_wedge(const DevGraph& g, const uint32_t
     }
     const uint32_t total = __shfl_sync(GMBE_FULL, inc, 31);
     const uint32_t excl = inc - deg;
-    for (uint32_t base = 0; base < total; base += 32) {
-      const uint32_t p = base + lane;
-      uint32_t lo = 0;
+    // GMBE_WEDGE_UNROLL chunks of 32 wedges per step (knob; 1 = default, 2/4/8 measured slower at
+    // N=1 and no better for 1/8 shards, profiles/r01_wedge_unroll_ab.txt): all their loads are in flight
+    // before the first callback (a lone heavy root is one warp's latency chain otherwise); the
+    // callbacks then run in the original chunk order, so the result is unchanged
+    for (uint32_t base = 0; base < total; base += 32 * GMBE_WEDGE_UNROLL) {
+      uint32_t vq[GMBE_WEDGE_UNROLL], iq[GMBE_WEDGE_UNROLL];
 #pragma unroll
-      for (int st = 16; st; st >>= 1) {
-        const uint32_t cand = lo + st;
-        const uint32_t e = __shfl_sync(GMBE_FULL, excl, cand & 31);
-        if (cand < 32 && e <= p) lo = cand;
+      for (int q = 0; q < GMBE_WEDGE_UNROLL; q++) {
+        const uint32_t p = base + 32 * q + lane;
+        uint32_t lo = 0;
+#pragma unroll
+        for (int st = 16; st; st >>= 1) {
+          const uint32_t cand = lo + st;
+          const uint32_t e = __shfl_sync(GMBE_FULL, excl, cand & 31);
+          if (cand < 32 && e <= p) lo = cand;
+        }
+        const uint32_t ob = __shfl_sync(GMBE_FULL, beg, lo);
+        const uint32_t oe = __shfl_sync(GMBE_FULL, excl, lo);
+        vq[q] = p < total ? g.adj_u[ob + p - oe] : 0;
+        iq[q] = b + lo;
       }
-      const uint32_t ob = __shfl_sync(GMBE_FULL, beg, lo);
-      const uint32_t oe = __shfl_sync(GMBE_FULL, excl, lo);
-      const bool act = p < total;
-      const uint32_t v = act ? g.adj_u[ob + p - oe] : 0;
-      f(b + lo, v, act);
+#pragma unroll
+      for (int q = 0; q < GMBE_WEDGE_UNROLL; q++)
+        if (base + 32 * q < total) f(iq[q], vq[q], base + 32 * q + lane < total);
     }
   }
 }
