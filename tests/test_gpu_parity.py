@@ -613,3 +613,34 @@ def test_cost_parts_full_config(gmbe, name, n):
         assert sum(r.nodes for r in rs) == gd["nodes"]
     finally:
         g.free()
+
+
+def test_cost_parts_and_cursor_edge_cases(gmbe):
+    """More parts than roots (empty parts), an empty graph, and a shared cursor over a graph with
+    fewer roots than the callers' warps."""
+    nu, nv = 5, 3
+    e = np.array([[0, 0], [1, 0], [1, 1], [2, 1], [3, 2], [4, 2], [4, 0]], np.uint32)
+    o = oracle.oracle_mbe(nu, nv, e)
+    g = gmbe.load(nu, nv, e)
+    try:
+        for n in (2, 3, 4, 8):
+            rs = [g.enumerate(part=(i, n), part_mode="cost") for i in range(n)]
+            assert sum(r.count for r in rs) == o.count
+            assert sum(r.checksum for r in rs) % (1 << 64) == o.checksum
+            assert sum(1 for r in rs if r.roots_run) <= nv
+        cur = gmbe.SharedCursor.create(0)
+        try:
+            a = g.enumerate(root_cursor=cur.slot_ptr(0))
+            b = g.enumerate(root_cursor=cur.slot_ptr(0))
+            assert (a.count, a.checksum) == (o.count, o.checksum) and b.count == 0
+        finally:
+            cur.close()
+    finally:
+        g.free()
+    g = gmbe.load(4, 4, np.zeros((0, 2), np.uint32))
+    try:
+        for n in (1, 3):
+            r = g.enumerate(part=(n - 1, n), part_mode="cost")
+            assert (r.count, r.checksum) == (0, 0)
+    finally:
+        g.free()
