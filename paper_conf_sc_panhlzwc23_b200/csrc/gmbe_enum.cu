@@ -2635,7 +2635,19 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   const bool want_out = o.out_ids != nullptr || sink != nullptr;
   const uint32_t rbuf_words = want_out ? (uint32_t)(wb + 64) : 0;
 
-  GMBE_CUDA_TRY(ensure(&W.arena, &W.arena_bytes, nwarps * arena_words * 4));
+  {
+    cudaError_t ae = ensure(&W.arena, &W.arena_bytes, nwarps * arena_words * 4);
+    // another process on this GPU may have taken memory since cudaMemGetInfo: halve the
+    // (free-memory-capped) dynamic region and retry, down to its floor
+    while (ae == cudaErrorMemoryAllocation && !o.arena_words && W.dyn > (1u << 16)) {
+      (void)cudaGetLastError();
+      W.dyn = std::max<uint64_t>(W.dyn / 2, 1u << 16);
+      W.dyn_capped = true;
+      arena_words = (3 * tmax + omax + 8 + W.dyn + 3) & ~3ull;
+      ae = ensure(&W.arena, &W.arena_bytes, nwarps * arena_words * 4);
+    }
+    GMBE_CUDA_TRY(ae);
+  }
   {
     const uint64_t sig[4] = {tmax, omax, arena_words, nwarps};
     if (!W.clean || std::memcmp(sig, W.layout, sizeof(sig)) != 0) {

@@ -532,9 +532,13 @@ def _ipc_worker(rank, world, port, name, q):
     torch.cuda.set_device(0)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        dr = gdist.DynamicRoots(rank, world, device=0)
         nu, nv, e = make_config(name)
         g = m.load(nu, nv, e)
+        for i in range(world):  # processes sharing one GPU size their workspaces in turn
+            if rank == i:
+                g.enumerate(part=(rank, world))
+            dist.barrier()
+        dr = gdist.DynamicRoots(rank, world, device=0)
         outs = []
         for _ in range(3):
             r, tot = dr.enumerate(g)
@@ -546,6 +550,9 @@ def _ipc_worker(rank, world, port, name, q):
         dist.barrier()
         if not rank:
             dr.close()
+    except Exception as ex:  # report instead of leaving the parent waiting on the queue
+        q.put((rank, False, "%s: %s" % (type(ex).__name__, ex), []))
+        raise
     finally:
         dist.destroy_process_group()
 
@@ -559,12 +566,15 @@ def test_dynamic_roots_two_processes_ipc(gmbe):
         s.bind(("127.0.0.1", 0))
         port = s.getsockname()[1]
     gd = _gold_cfg()["gh"]
+    g = gmbe.load(2, 2, np.array([[0, 0]], np.uint32))  # hand this process's idle workspace back
+    g.release_workspace()
+    g.free()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     ps = [ctx.Process(target=_ipc_worker, args=(r, 2, port, "gh", q)) for r in range(2)]
     for p in ps:
         p.start()
-    out = sorted(q.get(timeout=600) for _ in range(2))
+    out = sorted(q.get(timeout=300) for _ in range(2))
     for p in ps:
         p.join(timeout=120)
         assert p.exitcode == 0
