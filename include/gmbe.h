@@ -207,7 +207,8 @@ int gmbe_enumerate_stream(const gmbe_graph* g, const gmbe_opts* opts, gmbe_sink_
  *   open   : map another process's block on `device` (the current GPU of this process);
  *            *dptr = this process's pointer to slot 0.  EINVAL for NULL args, ECUDA if CUDA IPC or
  *            peer access is unavailable (the caller falls back to static parts).
- *   reset  : zero slot `slot` of the block at dptr, stream-ordered on `cuda_stream` (NULL = legacy).
+ *   reset  : zero slot `slot` of the block at dptr, stream-ordered on `cuda_stream` (NULL = legacy);
+ *            call with the device that owns (or maps) dptr current.  EINVAL: NULL dptr, bad slot.
  *   close  : unmap (opened) or free (created, owner = 1) the block.  NULL-safe. */
 enum { GMBE_CURSOR_SLOTS = 16, GMBE_IPC_HANDLE_BYTES = 64 };
 int gmbe_shared_cursor_create(int32_t device, uint64_t** dptr, void* ipc_handle);

@@ -70,3 +70,17 @@ def test_import_fails_loudly_without_library(tmp_path):
     r = subprocess.run([sys.executable, "-c", "import paper_conf_sc_panhlzwc23_b200"], cwd=tmp_path,
                        capture_output=True, text=True)
     assert r.returncode != 0 and "libgmbe.so is not built" in r.stderr
+
+
+def test_enum_constants_match_c(gmbe, tmp_path):
+    """The binding's copies of the header's enums (cursor slots, IPC handle size, part modes)."""
+    c = tmp_path / "en.c"
+    c.write_text('#include <stdio.h>\n#include "gmbe.h"\nint main(){printf("%d %d %d %d\\n",'
+                 ' GMBE_CURSOR_SLOTS, GMBE_IPC_HANDLE_BYTES, GMBE_PART_INTERLEAVE, GMBE_PART_COST);'
+                 'return 0;}')
+    exe = tmp_path / "en"
+    subprocess.check_call(["gcc", "-I", os.path.dirname(HDR), str(c), "-o", str(exe)])
+    got = list(map(int, subprocess.check_output([str(exe)]).split()))
+    assert got == [gmbe.CURSOR_SLOTS, gmbe.IPC_HANDLE_BYTES, gmbe.PART_MODE["interleave"],
+                   gmbe.PART_MODE["cost"]]
+    assert ctypes.sizeof(ctypes.c_uint64) * 16 == 128  # one cursor slot per 128-byte line (slot_ptr)
