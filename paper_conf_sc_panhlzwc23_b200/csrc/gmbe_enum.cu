@@ -1118,6 +1118,27 @@ __device__ __forceinline__ bool heavy(const Params& P, uint32_t l, uint32_t nC) 
   // the node count alone under-estimates the work (B200 addition, reading B4)
   return l > 64 && nC >= 2 && (unsigned long long)nC * ((l + 31) / 32) >= P.split_wide;
 }
+// Late-phase split (B200 addition): once GMBE_LATE_PCT % of the roots have been issued, the GPU is
+// about to drain, and a mid-size task started now would run alone in the tail -- so tasks above the
+// lower (GMBE_LATE_BH, GMBE_LATE_BS) thresholds split too.  Schedule only: the tree is unchanged.
+// Knob, off by default: measured +0.5-3% at N=1 and 3-5x slower on 1/8 root shards (a shard's
+// cursor passes the mark almost at once), profiles/r01_late_split_ab.txt.
+#ifndef GMBE_LATE_PCT
+#define GMBE_LATE_PCT 0
+#endif
+#ifndef GMBE_LATE_BH
+#define GMBE_LATE_BH 6
+#endif
+#ifndef GMBE_LATE_BS
+#define GMBE_LATE_BS 120
+#endif
+__device__ __forceinline__ bool late_heavy(const Params& P, uint32_t l, uint32_t nC) {
+  if (GMBE_LATE_PCT == 0 || !P.split) return false;
+  const unsigned long long h = min(l, nC);
+  if (h <= GMBE_LATE_BH || h * nC <= GMBE_LATE_BS) return false;
+  const unsigned long long c = ld_volatile(P.shared_cursor ? P.shared_cursor : &P.ctrl->root_cursor.v);
+  return 100ull * c >= (unsigned long long)GMBE_LATE_PCT * P.n_roots;
+}
 __device__ __forceinline__ bool heavy_wide(const Params& P, uint32_t l, uint32_t nC) {
   return P.split && l > 64 && nC >= 2 && (unsigned long long)nC * ((l + 31) / 32) >= P.split_wide;
 }
@@ -1753,7 +1774,7 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
   const uint32_t lane = lane_id();
   uint32_t* cur = top;
   uint32_t* sp = stack_lo;  // first free word
-  const bool split_mode = heavy(P, top[2], top[0]);
+  const bool split_mode = heavy(P, top[2], top[0]) || late_heavy(P, top[2], top[0]);
   if (split_mode) A.splits++;
   // register-resident DFS (one inline site): the whole task if its top has <= 32 candidates,
   // else every pushed child with <= 32 candidates
