@@ -166,9 +166,9 @@ def _dyn_worker(rank, world, port, fail_rank, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("fail_rank", [None, 1])
-def test_dynamic_roots_protocol(fail_rank):
-    world, port = 2, _free_port()
+@pytest.mark.parametrize("world,fail_rank", [(2, None), (2, 1), (3, None), (3, 2)])
+def test_dynamic_roots_protocol(world, fail_rank):
+    port = _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     ps = [ctx.Process(target=_dyn_worker, args=(r, world, port, fail_rank, q)) for r in range(world)]
