@@ -22,7 +22,15 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 DEFAULT_CONFIG = "gh_work"
-METRIC = "maximal bicliques/sec (Github-shaped)"
+METRIC = "maximal bicliques/sec (Github-shaped)"  # BASELINE.json's metric, on the default gh_work
+_SHAPES = {"gh": "Github", "yg": "YouTube", "bx": "BookCrossing", "dblp": "DBLP", "er": "Erdos-Renyi"}
+
+
+def _metric(config):
+    for k, v in _SHAPES.items():
+        if config.startswith(k):
+            return "maximal bicliques/sec (%s-shaped)" % v
+    return METRIC
 CTRL_BYTES = 1152  # sizeof(Ctrl): written and read back by gmbe_enumerate (static_assert in gmbe_enum.cu)
 
 
@@ -153,7 +161,7 @@ def run_reference(a):
         times.append(dt)
         counts.append(c)
     v = sum(counts) / sum(times)
-    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "bicliques/s",
+    line = {"impl": "reference", "metric": _metric(a.config), "value": v, "unit": "bicliques/s",
             "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup,
             "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
@@ -332,7 +340,7 @@ def main():
         if share and ws > 1:
             par += " [TEST: all ranks share GPU 0 over gloo; not a multi-GPU measurement]"
         line = {
-            "metric": METRIC, "value": count / (t_step * 1e-3), "unit": "bicliques/s",
+            "metric": _metric(a.config), "value": count / (t_step * 1e-3), "unit": "bicliques/s",
             "n_gpus": ws, "steps": a.steps, "warmup": a.warmup, "ms_per_step": t_step,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "u32", "data": "synthetic",
