@@ -34,7 +34,7 @@ enum {
   GMBE_EINVAL = -1,       /* bad argument: NULL pointer, id >= n_u / n_v, bad option value */
   GMBE_ENOMEM = -2,       /* device allocation failed (nothing leaks, the graph stays valid) */
   GMBE_ECUDA = -3,        /* a CUDA runtime call or kernel failed */
-  GMBE_EUNSUPPORTED = -4, /* input beyond implemented limits (n_edges >= 2^32, ids >= 2^31) */
+  GMBE_EUNSUPPORTED = -4, /* input beyond implemented limits (n_edges >= 2^31, |U| or |V| >= 2^31) */
   GMBE_EINTERNAL = -5     /* a device-side capacity was exceeded (workspace too small) */
 };
 
@@ -59,7 +59,7 @@ typedef struct {
  *                device memory if opts->edges_on_device.  Read during the call only.
  *   out        : receives the new graph handle (free with gmbe_free_graph).
  * Errors: EINVAL (NULL out, NULL edges with n_edges>0, id out of range), EUNSUPPORTED
- * (n_edges >= 2^32 or n_u, n_v >= 2^31), ENOMEM, ECUDA. */
+ * (n_edges >= 2^31 or n_u, n_v >= 2^31), ENOMEM, ECUDA. */
 int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* edges_uv, uint64_t n_edges,
                         const gmbe_load_opts* opts, gmbe_graph** out);
 
@@ -96,7 +96,13 @@ typedef struct {
   uint32_t part_count;    /*   r % part_count == part_index (0 = 1 part); shards partition the
                                output, so counts / checksums add (mod 2^64) across parts */
   uint32_t reserved0;     /* debug bits for tests / experiments (0 in production use) */
-  uint32_t reserved1;     /* must be 0 */
+  uint32_t scheduler;     /* GMBE_SCHED_*: how root tasks map to the GPU (Sec 4.3):
+                             TASK (0, default) = GMBE's load-aware task-centric scheme (Alg 4);
+                             WARP (1) = GMBE-WARP, one warp per Alg 3 task, no splitting, one node
+                             per warp step; BLOCK (2) = GMBE-BLOCK, one thread block per Alg 3 task,
+                             no splitting, every node generated by the whole block.  The variants of
+                             Sec 6.3 (Fig 8/9); the result and the canonical-tree counters are the
+                             same in all three. */
   /* Optional bounded output (device-accessible memory: device or mapped pinned host).
    * Record = [|L|, |R|, L ids (caller U ids), R ids (caller V ids)], order within a record and of
    * records unspecified; out_offsets[i] = word offset of record i in out_ids.  A full buffer is
@@ -158,6 +164,7 @@ typedef struct {
 } gmbe_opts;
 
 enum { GMBE_PART_INTERLEAVE = 0, GMBE_PART_COST = 1 };
+enum { GMBE_SCHED_TASK = 0, GMBE_SCHED_WARP = 1, GMBE_SCHED_BLOCK = 2 };
 
 typedef struct {
   uint64_t count;         /* maximal bicliques enumerated (this shard) */
@@ -190,7 +197,8 @@ int gmbe_enumerate(const gmbe_graph* g, const gmbe_opts* opts, gmbe_result* out)
  * `words` is valid only during the call.  count / checksum / counters are as in gmbe_enumerate;
  * result.n_written = records delivered (== count).  opts must not carry out_offsets / out_ids.
  * Errors: as gmbe_enumerate; EINVAL (NULL sink, bounded buffers given, the sink returned non-zero
- * -- the remaining records are drained but not delivered); EINTERNAL (a producer waited > 20 s). */
+ * -- the remaining records are drained but not delivered).  A slow sink only slows the kernel down
+ * (producers wait for room; there is no timeout), so the sink must eventually return. */
 typedef int (*gmbe_sink_fn)(const uint32_t* words, uint64_t n_words, uint64_t n_records, void* user);
 int gmbe_enumerate_stream(const gmbe_graph* g, const gmbe_opts* opts, gmbe_sink_fn sink, void* user,
                           uint64_t ring_words, gmbe_result* out);
@@ -207,7 +215,8 @@ int gmbe_enumerate_stream(const gmbe_graph* g, const gmbe_opts* opts, gmbe_sink_
  *   open   : map another process's block on `device` (the current GPU of this process);
  *            *dptr = this process's pointer to slot 0.  EINVAL for NULL args, ECUDA if CUDA IPC or
  *            peer access is unavailable (the caller falls back to static parts).
- *   reset  : zero slot `slot` of the block at dptr, stream-ordered on `cuda_stream` (NULL = legacy);
+ *   reset  : zero slot `slot` of the block at dptr on `cuda_stream` (NULL = legacy) and wait for it
+ *            (synchronous, so the zero is visible to every stream and process when it returns);
  *            call with the device that owns (or maps) dptr current.  EINVAL: NULL dptr, bad slot.
  *   close  : unmap (opened) or free (created, owner = 1) the block.  NULL-safe. */
 enum { GMBE_CURSOR_SLOTS = 16, GMBE_IPC_HANDLE_BYTES = 64 };

@@ -44,7 +44,7 @@ def _load():
         f = _lib.oracle_mbe
         u32, u64, ptr = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p
         f.argtypes = [u32, u32, ptr, u64, ctypes.c_int, ctypes.c_int, u32, u32, ctypes.c_int,
-                      ptr, u64, ptr, u64, ptr, ctypes.POINTER(_Res)]
+                      ptr, u64, ptr, u64, ptr, ptr, ptr, ctypes.POINTER(_Res)]
         f.restype = ctypes.c_int
     return _lib
 
@@ -63,11 +63,15 @@ class OracleResult:
     algo_bytes_cand: int = 0
     bicliques: list = None      # list of (tuple(L), tuple(R)) in caller ids, if requested
     per_root_count: np.ndarray = None
+    per_root_ns: np.ndarray = None
 
 
 def oracle_mbe(n_u, n_v, edges, order="degree", prune=True, shard=(0, 1), check_closure=False,
-               records=False, rec_cap=1 << 20, ids_cap=1 << 24, per_root=False):
-    """Run the oracle on edge list `edges` (uint32 [m,2], rows (u,v), caller ids)."""
+               records=False, rec_cap=1 << 20, ids_cap=1 << 24, per_root=False, root_mask=None,
+               root_times=False):
+    """Run the oracle on edge list `edges` (uint32 [m,2], rows (u,v), caller ids).
+    root_mask: optional bool array over the internal V side (the smaller side; caller V unless
+    n_u < n_v): only those roots are enumerated.  root_times: also return per-root wall ns."""
     lib = _load()
     e = np.ascontiguousarray(np.asarray(edges, dtype=np.uint32).reshape(-1, 2))
     res = _Res()
@@ -77,12 +81,20 @@ def oracle_mbe(n_u, n_v, edges, order="degree", prune=True, shard=(0, 1), check_
         ids = np.zeros(ids_cap, np.uint32)
     nv_int = n_u if n_u < n_v else n_v
     prc = np.zeros(max(nv_int, 1), np.uint64) if per_root else None
+    msk = None
+    if root_mask is not None:
+        msk = np.ascontiguousarray(np.asarray(root_mask, dtype=np.uint8))
+        if len(msk) != nv_int:
+            raise ValueError("root_mask: length %d != |internal V| %d" % (len(msk), nv_int))
+    rns = np.zeros(max(nv_int, 1), np.uint64) if root_times else None
     rc = lib.oracle_mbe(n_u, n_v, e.ctypes.data if len(e) else None, len(e),
                         0 if order == "degree" else 1, 1 if prune else 0, shard[0], shard[1],
                         1 if check_closure else 0,
                         offs.ctypes.data if records else None, rec_cap if records else 0,
                         ids.ctypes.data if records else None, ids_cap if records else 0,
-                        prc.ctypes.data if per_root else None, ctypes.byref(res))
+                        prc.ctypes.data if per_root else None,
+                        msk.ctypes.data if msk is not None and len(msk) else None,
+                        rns.ctypes.data if root_times else None, ctypes.byref(res))
     if rc != 0:
         raise ValueError("oracle_mbe: invalid arguments")
     out = OracleResult(res.count, res.checksum, res.roots_run, res.nodes, res.nonmax,
@@ -92,6 +104,8 @@ def oracle_mbe(n_u, n_v, edges, order="degree", prune=True, shard=(0, 1), check_
         out.bicliques = decode_records(offs[:res.n_written], ids)
     if per_root:
         out.per_root_count = prc[:nv_int]
+    if root_times:
+        out.per_root_ns = rns[:nv_int]
     return out
 
 

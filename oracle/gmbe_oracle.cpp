@@ -30,6 +30,7 @@
 #include <cstdint>
 #include <cstring>
 #include <pthread.h>
+#include <time.h>
 #include <vector>
 
 namespace {
@@ -78,6 +79,8 @@ struct Options {
   uint32_t* rec_ids;
   uint64_t ids_cap;
   uint64_t* per_root_count;
+  const uint8_t* root_mask;  // optional: run only the roots v (internal V id) with root_mask[v] != 0
+  uint64_t* per_root_ns;     // optional: wall-clock ns spent on each root (internal V id)
 };
 
 struct Result {
@@ -265,8 +268,20 @@ struct Oracle {
   void run() {
     std::vector<uint32_t> by_rank(nV);
     for (uint32_t v = 0; v < nV; v++) by_rank[rank[v]] = v;
-    for (uint32_t rk = 0; rk < nV; rk++)
-      if (rk % opt.shard_n == opt.shard_i) run_root(by_rank[rk]);
+    for (uint32_t rk = 0; rk < nV; rk++) {
+      const uint32_t v = by_rank[rk];
+      if (rk % opt.shard_n != opt.shard_i) continue;
+      if (opt.root_mask && !opt.root_mask[v]) continue;
+      if (opt.per_root_ns) {
+        timespec t0, t1;
+        clock_gettime(CLOCK_MONOTONIC, &t0);
+        run_root(v);
+        clock_gettime(CLOCK_MONOTONIC, &t1);
+        opt.per_root_ns[v] += (uint64_t)((t1.tv_sec - t0.tv_sec) * 1000000000LL + (t1.tv_nsec - t0.tv_nsec));
+      } else {
+        run_root(v);
+      }
+    }
   }
 };
 
@@ -292,10 +307,14 @@ typedef struct {
 // order: 0 ascending degree (ties: ascending id, reading A8), 1 identity.
 // per_root_count (optional): indexed by the internal-V id of the root (caller's V id unless the
 //   sides were swapped, in which case the caller's U id).
+// root_mask (optional, same indexing): enumerate only the roots with root_mask[v] != 0 (a root
+//   sample for timing; like shards, masks partition the output).  per_root_ns (optional, same
+//   indexing): wall-clock nanoseconds spent on each root's tree (timing only).
 int oracle_mbe(uint32_t n_u, uint32_t n_v, const uint32_t* edges, uint64_t n_edges, int order,
                int prune, uint32_t shard_i, uint32_t shard_n, int check_closure,
                uint64_t* rec_offsets, uint64_t rec_cap, uint32_t* rec_ids, uint64_t ids_cap,
-               uint64_t* per_root_count, oracle_result* out) {
+               uint64_t* per_root_count, const uint8_t* root_mask, uint64_t* per_root_ns,
+               oracle_result* out) {
   if (!out || shard_n == 0 || shard_i >= shard_n || (n_edges && !edges)) return -1;
   for (uint64_t e = 0; e < n_edges; e++)
     if (edges[2 * e] >= n_u || edges[2 * e + 1] >= n_v) return -1;
@@ -328,7 +347,7 @@ int oracle_mbe(uint32_t n_u, uint32_t n_v, const uint32_t* edges, uint64_t n_edg
   o.rank.assign(o.nV, 0);
   for (uint32_t r = 0; r < o.nV; r++) o.rank[by_rank[r]] = r;
   o.opt = Options{order, prune, shard_i, shard_n, check_closure, rec_offsets, rec_cap,
-                  rec_ids, ids_cap, per_root_count};
+                  rec_ids, ids_cap, per_root_count, root_mask, per_root_ns};
   if (!rec_offsets || !rec_ids) o.opt.rec_offsets = nullptr, o.opt.rec_ids = nullptr;
   std::memset(&o.res, 0, sizeof(o.res));
   // recursion depth <= min(|L|,|C|) <= Delta(V): run on a thread with a large stack

@@ -33,6 +33,7 @@ EXPORTS = ("gmbe_load_bipartite", "gmbe_graph_info_get", "gmbe_free_graph", "gmb
            "gmbe_shared_cursor_reset", "gmbe_shared_cursor_close")
 CURSOR_SLOTS, IPC_HANDLE_BYTES = 16, 64
 PART_MODE = {"interleave": 0, "cost": 1}
+SCHEDULER = {"task": 0, "warp": 1, "block": 2}  # GMBE (Alg 4), GMBE-WARP, GMBE-BLOCK
 
 _u32, _i32, _u64, _vp = ctypes.c_uint32, ctypes.c_int32, ctypes.c_uint64, ctypes.c_void_p
 
@@ -51,7 +52,7 @@ class GraphInfo(ctypes.Structure):
 class Opts(ctypes.Structure):
     _fields_ = [("struct_size", _u32), ("no_prune", _u32), ("no_split", _u32), ("bound_height", _u32),
                 ("bound_size", _u32), ("warps_per_sm", _u32), ("part_index", _u32),
-                ("part_count", _u32), ("reserved0", _u32), ("reserved1", _u32),
+                ("part_count", _u32), ("reserved0", _u32), ("scheduler", _u32),
                 ("out_offsets", _vp), ("out_offsets_cap", _u64), ("out_ids", _vp),
                 ("out_ids_cap", _u64), ("per_root_count", _vp), ("per_root_cycles", _vp), ("phase_cycles", _vp), ("timeline", _vp), ("timeline_cap", _u64),
                 ("arena_words", _u64),
@@ -144,10 +145,17 @@ class Result:
     timeline: np.ndarray = field(default=None, repr=False)
 
 
+CUDA_STREAM_LEGACY = 0x1  # cudaStreamLegacy: the legacy default stream as an explicit handle
+
+
 def _stream_ptr(stream):
+    """cudaStream_t of a torch stream (or a raw handle).  torch's default stream has handle 0, which
+    the library reads as "no stream given" (its own non-blocking stream, NOT ordered after torch's
+    work), so it is passed as cudaStreamLegacy instead."""
     if stream is None:
         return None
-    return int(getattr(stream, "cuda_stream", stream))
+    h = int(getattr(stream, "cuda_stream", stream))
+    return h if h else CUDA_STREAM_LEGACY
 
 
 class Graph:
@@ -168,10 +176,11 @@ class Graph:
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
                   per_root=False, root_cycles=False, phases=False, timeline=0, debug=0, thr_min=0, split_wide=0, arena_words=0, pool_words=0, queue_cap=0, stream=None,
-                  root_cursor=None, part_mode="interleave"):
+                  root_cursor=None, part_mode="interleave", scheduler="task"):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them.
         root_cursor: device address (int) of a shared root-cursor slot (SharedCursor.slot_ptr).
-        part_mode: how `part` splits the roots -- "interleave" (degree rank mod N) or "cost" (N4)."""
+        part_mode: how `part` splits the roots -- "interleave" (degree rank mod N) or "cost" (N4).
+        scheduler: "task" (GMBE, default), "warp" (GMBE-WARP) or "block" (GMBE-BLOCK), Sec 4.3."""
         o = Opts()
         o.struct_size = ctypes.sizeof(Opts)
         o.no_prune = 0 if prune else 1
@@ -184,6 +193,7 @@ class Graph:
         o.thr_min, o.split_wide = thr_min, split_wide
         o.root_cursor = root_cursor
         o.part_mode = PART_MODE[part_mode]
+        o.scheduler = SCHEDULER[scheduler]
         bufs = None
         if records:
             import torch
@@ -207,7 +217,9 @@ class Graph:
         tl = None
         if timeline:
             import torch
-            tl = torch.zeros(1 + 4 * timeline, dtype=torch.int64, device=torch.device("cuda", self.info()["device"]))
+            tdev = torch.device("cuda", self.info()["device"])
+            tl = torch.zeros(1 + 4 * timeline, dtype=torch.int64, device=tdev)
+            torch.cuda.current_stream(tdev).synchronize()  # the fill is on torch's stream, not the library's
             o.timeline, o.timeline_cap = tl.data_ptr(), 1 + 4 * timeline
         phc = None
         if phases:
@@ -350,15 +362,23 @@ def load(n_u, n_v, edges, order="degree", device=None, stream=None):
     lo.order = ORDER[order]
     keep = None
     if hasattr(edges, "is_cuda") and edges.is_cuda:
+        import torch
         e = edges.contiguous()
-        assert e.element_size() == 4
+        if e.element_size() != 4:
+            raise TypeError("device edges must be a 32-bit integer tensor")
         ptr, m = e.data_ptr(), e.numel() // 2
         lo.edges_on_device = 1
         if device is None:
             lo.device = e.device.index
+        if stream is None:
+            # the edges were produced (or made contiguous) on torch's current stream: build on it
+            lo.cuda_stream = _stream_ptr(torch.cuda.current_stream(e.device))
         keep = e
     else:
-        e = np.ascontiguousarray(np.asarray(edges).astype(np.uint32, copy=False).reshape(-1, 2))
+        a = np.asarray(edges)
+        if a.dtype == np.int32:
+            a = a.view(np.uint32)  # zero-copy (e.g. a pinned int32 buffer stays pinned)
+        e = np.ascontiguousarray(a.astype(np.uint32, copy=False).reshape(-1, 2))
         ptr, m = (e.ctypes.data if len(e) else None), len(e)
         keep = e
     h = _vp()

@@ -4,7 +4,7 @@ import subprocess
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 SRC = [os.path.join(HERE, "csrc", f) for f in ("gmbe_api.cu", "gmbe_graph.cu", "gmbe_enum.cu")]
-DEPS = SRC + [os.path.join(HERE, "csrc", "gmbe_internal.cuh"),
+DEPS = SRC + [os.path.join(HERE, "csrc", "gmbe_internal.cuh"), os.path.join(HERE, "csrc", "gmbe_block.cuh"),
               os.path.join(os.path.dirname(HERE), "include", "gmbe.h")]
 LIB = os.path.join(HERE, "libgmbe.so")
 LIB_PROF = os.path.join(HERE, "libgmbe_prof.so")  # phase-profiling variant (-DGMBE_PROFILE)

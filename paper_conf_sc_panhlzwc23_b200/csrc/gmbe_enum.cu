@@ -89,7 +89,8 @@ struct Params {
   uint32_t debug;  // opts.reserved0 bits (tests / experiments): 4 = no donation, 8 = donate whenever possible,
                    // 16 = no thread-level tier (run_thr), 32 = path statistics into ctrl.phase,
                    // 64 = no suffix-mode roots, 128 = every root in suffix mode, 256 = no dense-mode roots,
-                   // 512 = dense mode whenever the table can hold it
+                   // 512 = dense mode whenever the table can hold it, 1024 = build the roots only
+                   // (timing experiments: no subtree is walked, the result is incomplete)
   uint32_t donate;  // dynamic donation to idle warps (donate_reg)
   uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.thr_min)
   uint32_t split_wide;   // wide-universe split threshold on |C|·⌈|L|/32⌉ (opts.split_wide)
@@ -571,14 +572,13 @@ __device__ bool rec_open(const Params& P, unsigned long long need, RecOut& O, un
     const unsigned long long pos = atomicAdd(&P.ctrl->out_ids, need + 1);
     atomicAdd(&P.ctrl->out_rec, 1ull);
     const unsigned long long end = pos + need + 1, cap = P.smask + 1;
-    unsigned long long t0 = 0;
-    while (end - ld_volatile(&P.ctrl->stream_tail) > cap) {  // ring full: back-pressure
+    // ring full: back-pressure.  No timeout -- a slow consumer only slows the call; the wait ends
+    // when the consumer frees room, or at once when the host raises its abort word
+    while (end - ld_volatile(&P.ctrl->stream_tail) > cap) {
       const unsigned long long t = *(volatile const unsigned long long*)P.stail;  // host memory
       atomicMax(&P.ctrl->stream_tail, t);
       if (end - t <= cap) break;
-      const unsigned long long now = globaltimer_ns();
-      if (!t0) t0 = now;
-      if (now - t0 > 20000000000ull) {  // the consumer is gone: give up (the call reports an error)
+      if (*(volatile const unsigned long long*)(P.stail + 1)) {  // the consumer gave up
         atomicOr(&P.ctrl->error, kErrStream);
         return false;
       }
@@ -1594,6 +1594,9 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
   uint32_t C = cand_all, next = 0, Rm = 0, d = 0, dmask = 0;
   uint32_t bd = 0;  // tree depth (below the job's top) of this lane's level 0
   uint32_t n_nodes = 0, n_nonmax = 0, n_count = 0;
+#ifdef GMBE_STATS
+  unsigned long long st_l = 0, st_lp = 0, st_later = 0, st_push = 0;  // path statistics (debug 32)
+#endif
   unsigned long long abytes = 0, cks = 0;
 #if GMBE_DONATE
   uint32_t tick = 0, hflag = 0;  // hflag: lane 0's in-flight read of ctrl.hungry (consumed 4 steps later)
@@ -1706,6 +1709,13 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     if (P.prune) C &= ~pr;
     n_nodes++;
     abytes += lc + ksum;
+#ifdef GMBE_STATS
+    if (P.debug & 32) {
+      st_l += __popcll(L);
+      st_lp += lc;
+      st_later += __popc(later);
+    }
+#endif
     const uint32_t rl = rlen0 + __popc(Rm) + 1 + __popc(ab);
     // maximality (Alg 2 L14): |Γ(L')| == |R'|; the emission's SL = Σ_{u∈L'} hU(u) on the same pass
     bool maximal;
@@ -1745,6 +1755,9 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     if (P.per_root) atomicAdd(P.per_root + T.root, 1ull);
     if (T.rlist && (P.out_ids || P.sring)) write_record_thr(P, T, ts, lp, lc, rlen0, rmn, rl);
     if (!cd) continue;
+#ifdef GMBE_STATS
+    if (P.debug & 32) st_push++;
+#endif
     // push (Alg 2 L16)
     stk[d].L = L;
     stk[d].SR = SR;
@@ -1759,6 +1772,20 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     Rm = rmn;
     next = 0;
   }
+#ifdef GMBE_STATS
+  if (P.debug & 32) {
+    st_l = warp_sum64(st_l);
+    st_lp = warp_sum64(st_lp);
+    st_later = warp_sum64(st_later);
+    st_push = warp_sum64(st_push);
+    if (lane == 0) {
+      atomicAdd(&P.ctrl->phase[8], st_l);
+      atomicAdd(&P.ctrl->phase[9], st_lp);
+      atomicAdd(&P.ctrl->phase[10], st_later);
+      atomicAdd(&P.ctrl->phase[11], st_push);
+    }
+  }
+#endif
   A.nodes += warp_sum(n_nodes);
   A.nonmax += warp_sum(n_nonmax);
   A.count += warp_sum(n_count);
@@ -2388,6 +2415,7 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
         kind = 0;
         item = rk;
         if (run_root(P, rk, M, A, Tc, &top, &lo)) lmap = top[2];
+        if (P.debug & 1024) top = nullptr;  // experiments: root construction only (no subtrees)
         tl_l = P.timeline ? P.g.off_v[rk + 1] - P.g.off_v[rk] : 0;
       } else {
         if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
@@ -2435,6 +2463,8 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
   }
 }
 
+#include "gmbe_block.cuh"  // GMBE-BLOCK (block-centric ablation variant)
+
 // ---------------------------------------------------------------- host side
 struct Workspace {
   int device = -1;
@@ -2444,7 +2474,7 @@ struct Workspace {
   bool clean = false;
   uint64_t tmax = 0, omax = 0, dyn = 0, nwarps = 0, pool_auto = 0;  // cached sizing
   bool dyn_capped = false;
-  int sms = 0, bps_max = 0;
+  int sms = 0, bps_max = 0, bps_max_blk = 0;
   void* pool = nullptr;
   size_t pool_bytes = 0;
   void* rings = nullptr;
@@ -2571,6 +2601,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   if (o.part_index >= parts) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: part_index >= part_count");
   if (o.part_mode > GMBE_PART_COST || o.reserved2)
     return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: bad part_mode / reserved2");
+  if (o.scheduler > GMBE_SCHED_BLOCK) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: bad scheduler");
   if (o.root_cursor && parts > 1)
     return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: root_cursor needs part_count <= 1");
   if ((o.out_offsets == nullptr) != (o.out_ids == nullptr))
@@ -2591,12 +2622,14 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   if (W.sms == 0) {  // per-device constants, queried once per workspace
     GMBE_CUDA_TRY(cudaDeviceGetAttribute(&W.sms, cudaDevAttrMultiProcessorCount, G->device));
     GMBE_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&W.bps_max, k_enum, 32 * kWpb, 0));
+    GMBE_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&W.bps_max_blk, k_enum_block, kBlkThreads, 0));
   }
+  const bool block_mode = o.scheduler == GMBE_SCHED_BLOCK;
   uint32_t wps = o.warps_per_sm ? o.warps_per_sm : 64;
   if (wps < kWpb) wps = kWpb;
   if (wps > 64) wps = 64;
   uint32_t bps = wps / kWpb;
-  if ((int)bps > W.bps_max) bps = W.bps_max;
+  if ((int)bps > (block_mode ? W.bps_max_blk : W.bps_max)) bps = block_mode ? W.bps_max_blk : W.bps_max;
   if (bps < 1) bps = 1;
   const uint32_t blocks = (uint32_t)W.sms * bps;
   const uint64_t nwarps = (uint64_t)blocks * kWpb;
@@ -2612,8 +2645,19 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   const uint64_t dyn_want = o.arena_words ? o.arena_words
                                           : (uint64_t)g.rec_bound * 4 + 4 * wb + 2 * cols_bound + (1u << 18);
   uint64_t arena_words;
-  if (W.arena && W.nwarps == nwarps && W.tmax >= tmax && W.omax >= omax &&
-      (W.dyn >= dyn_want || (!o.arena_words && W.dyn_capped))) {
+  bool reuse = W.arena && W.nwarps == nwarps && W.tmax >= tmax && W.omax >= omax &&
+               (W.dyn >= dyn_want || (!o.arena_words && W.dyn_capped));
+  if (reuse && W.dyn < dyn_want) {
+    // a layout capped by free memory at an earlier call: re-size if there is more room now
+    size_t fr = 0, tot = 0;
+    GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
+    fr += W.arena_bytes;
+    const uint64_t fixed = 3 * W.tmax + W.omax + 8;
+    const uint64_t cap_total = (uint64_t)(fr * 0.5) / 4 / nwarps;
+    const uint64_t cap_now = cap_total > fixed ? cap_total - fixed : 0;
+    if (cap_now > W.dyn + W.dyn / 8) reuse = false;
+  }
+  if (reuse) {
     tmax = W.tmax;
     omax = W.omax;
     arena_words = W.layout[2];
@@ -2712,7 +2756,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
     P.issue = (const uint32_t*)sb;
   }
   P.prune = o.no_prune ? 0 : 1;
-  P.split = o.no_split ? 0 : 1;
+  P.split = o.no_split || o.scheduler != GMBE_SCHED_TASK ? 0 : 1;  // WARP / BLOCK: Alg 3 tasks, no split
   P.bound_height = o.bound_height ? o.bound_height : 10;   // paper: 20; retuned for B200
   P.bound_size = o.bound_size ? o.bound_size : 500;     // paper: 1500; scripts/sweep.py
   P.hu_side = g.swapped ? 1 : 0;
@@ -2749,7 +2793,8 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
       W.sring_words = words;
       W.sring_dirty = false;
     }
-    *(volatile unsigned long long*)(W.sring_h + words + 16) = 0;  // consumer tail
+    // consumer words after the ring: tail, abort (rec_open's back-pressure wait)
+    for (int k = 0; k < 2; k++) *(volatile unsigned long long*)(W.sring_h + words + 16 + 2 * k) = 0;
     P.sring = W.sring_d;
     P.smask = words - 1;
     P.stail = (const unsigned long long*)(W.sring_d + words + 16);
@@ -2758,7 +2803,8 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   P.per_root_cycles = o.per_root_cycles ? (unsigned long long*)W.per_root_cyc : nullptr;
   P.profile = o.phase_cycles ? 1 : 0;
   P.debug = o.reserved0;
-  P.donate = (o.reserved0 & 4) ? 0 : 1;
+  P.donate = (o.reserved0 & 4) || o.scheduler != GMBE_SCHED_TASK ? 0 : 1;
+  if (o.scheduler == GMBE_SCHED_WARP) P.debug |= 16;  // one warp per node: no thread-level tier
   P.thr_min_est = o.thr_min ? o.thr_min : GMBE_THR_MIN_EST;
   P.split_wide = o.split_wide ? o.split_wide : GMBE_SPLIT_WIDE;
   P.timeline = (unsigned long long*)o.timeline;
@@ -2776,7 +2822,11 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   GMBE_CUDA_TRY(cudaEventCreate(&e0));
   GMBE_CUDA_TRY(cudaEventCreate(&e1));
   GMBE_CUDA_TRY(cudaEventRecord(e0, s));
-  if (P.n_roots > 0) k_enum<<<blocks, 32 * kWpb, 0, s>>>(P), gmbe_note_launch();
+  if (P.n_roots > 0) {
+    if (block_mode) k_enum_block<<<blocks, kBlkThreads, 0, s>>>(P);
+    else k_enum<<<blocks, 32 * kWpb, 0, s>>>(P);
+    gmbe_note_launch();
+  }
   const cudaError_t le = cudaGetLastError();
   GMBE_CUDA_TRY(cudaEventRecord(e1, s));
   GMBE_CUDA_TRY(le);
@@ -2787,6 +2837,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
     // words, then advance the tail the producers wait on
     volatile uint32_t* R = W.sring_h;
     volatile unsigned long long* tail = (volatile unsigned long long*)(W.sring_h + W.sring_words + 16);
+    volatile unsigned long long* abort_word = tail + 1;  // raised if this consumer stops draining
     const uint64_t mask = W.sring_words - 1;
     std::vector<uint32_t> batch;
     uint64_t c = 0, nb = 0, final_pos = ~0ull;
@@ -2834,6 +2885,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
         failed = hc2.error != 0;
         done = true;
       } else if (q != cudaErrorNotReady) {
+        *abort_word = 1;  // producers waiting on a full ring stop at once
         GMBE_CUDA_TRY(q);
       }
     }
@@ -2926,7 +2978,10 @@ extern "C" int gmbe_shared_cursor_open(const void* ipc_handle, int32_t device, u
 
 extern "C" int gmbe_shared_cursor_reset(uint64_t* dptr, uint32_t slot, void* cuda_stream) {
   if (!dptr || slot >= GMBE_CURSOR_SLOTS) return gmbe_set_error(GMBE_EINVAL, "gmbe_shared_cursor_reset: bad argument");
+  // synchronous: the zero must have landed before any rank can start the call that uses the slot,
+  // whatever stream that call runs on
   GMBE_CUDA_TRY(cudaMemsetAsync(dptr + 16 * slot, 0, 8, (cudaStream_t)cuda_stream));
+  GMBE_CUDA_TRY(cudaStreamSynchronize((cudaStream_t)cuda_stream));
   return GMBE_OK;
 }
 

@@ -185,8 +185,9 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   if (!out) return gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: out is NULL");
   *out = nullptr;
   if (n_edges && !edges_uv) return gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: edges is NULL");
-  if (n_edges >= (1ull << 32) || n_u >= (1u << 31) || n_v >= (1u << 31))
-    return gmbe_set_error(GMBE_EUNSUPPORTED, "gmbe_load_bipartite: n_edges >= 2^32 or |U|,|V| >= 2^31");
+  // CUB's sorts / selects take int item counts: keep every count below 2^31
+  if (n_edges >= (1ull << 31) || n_u >= (1u << 31) || n_v >= (1u << 31))
+    return gmbe_set_error(GMBE_EUNSUPPORTED, "gmbe_load_bipartite: n_edges >= 2^31 or |U|,|V| >= 2^31");
   gmbe_load_opts o{};
   o.device = -1;
   if (opts) {

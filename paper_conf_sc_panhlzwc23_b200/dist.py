@@ -95,7 +95,12 @@ class DynamicRoots:
         else:
             agreed = self.cursor is not None
         if not agreed:
-            if self.cursor is not None:
+            # ranks that mapped the owner's block unmap it first; only then may the owner free it
+            if self.cursor is not None and rank != 0:
+                self.cursor.close()
+            if world > 1:
+                dist.barrier(group=group)
+            if self.cursor is not None and rank == 0:
                 self.cursor.close()
             self.cursor = None
         self.error = None if agreed else str(err or "a peer rank could not map the cursor")

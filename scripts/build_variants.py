@@ -20,8 +20,8 @@ def one(spec):
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode:
         return name + " FAILED\n" + r.stderr[-3000:]
-    lines = [l for l in (r.stdout + r.stderr).splitlines() if "k_enum" in l or "spill" in l or "Used" in l]
-    ke = [i for i, l in enumerate(lines) if "Function properties" in l and "k_enum" in l]
+    lines = [l for l in (r.stdout + r.stderr).splitlines() if "6k_enumEN" in l or "spill" in l or "Used" in l]
+    ke = [i for i, l in enumerate(lines) if "Function properties" in l and "6k_enumEN" in l]
     info = " | ".join(lines[ke[0] + 1: ke[0] + 3]) if ke else ""
     return "%s: %s" % (name, info)
 

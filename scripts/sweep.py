@@ -14,7 +14,7 @@ for spec in sys.argv[2:]:
     kw = {}
     for a in filter(None, spec.split(",")):
         k, v = a.split("=")
-        kw[k] = int(v)
+        kw[k] = int(v) if v.lstrip("-").isdigit() else v
     ts = []
     for _ in range(3):
         r = g.enumerate(**kw)

@@ -73,14 +73,17 @@ def test_import_fails_loudly_without_library(tmp_path):
 
 
 def test_enum_constants_match_c(gmbe, tmp_path):
-    """The binding's copies of the header's enums (cursor slots, IPC handle size, part modes)."""
+    """The binding's copies of the header's enums (cursor slots, IPC handle size, part modes,
+    schedulers)."""
     c = tmp_path / "en.c"
     c.write_text('#include <stdio.h>\n#include "gmbe.h"\nint main(){printf("%d %d %d %d\\n",'
                  ' GMBE_CURSOR_SLOTS, GMBE_IPC_HANDLE_BYTES, GMBE_PART_INTERLEAVE, GMBE_PART_COST);'
+                 'printf("%d %d %d\\n", GMBE_SCHED_TASK, GMBE_SCHED_WARP, GMBE_SCHED_BLOCK);'
                  'return 0;}')
     exe = tmp_path / "en"
     subprocess.check_call(["gcc", "-I", os.path.dirname(HDR), str(c), "-o", str(exe)])
     got = list(map(int, subprocess.check_output([str(exe)]).split()))
     assert got == [gmbe.CURSOR_SLOTS, gmbe.IPC_HANDLE_BYTES, gmbe.PART_MODE["interleave"],
-                   gmbe.PART_MODE["cost"]]
+                   gmbe.PART_MODE["cost"], gmbe.SCHEDULER["task"], gmbe.SCHEDULER["warp"],
+                   gmbe.SCHEDULER["block"]]
     assert ctypes.sizeof(ctypes.c_uint64) * 16 == 128  # one cursor slot per 128-byte line (slot_ptr)

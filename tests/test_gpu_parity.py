@@ -654,3 +654,165 @@ def test_cost_parts_and_cursor_edge_cases(gmbe):
             assert (r.count, r.checksum) == (0, 0)
     finally:
         g.free()
+
+
+# ---------------------------------------------------------------- stream ordering of device edges
+def test_device_edges_computed_on_torch_stream(gmbe):
+    """Edges produced by torch kernels (here a non-contiguous view that load() must copy, after a
+    computation on torch's current stream) are read by the graph build only after that work: the
+    binding builds on torch's current stream (the default stream is passed as cudaStreamLegacy)."""
+    import torch
+    gd = _gold_cfg()["gh"]
+    nu, nv, e = make_config("gh")
+    for rep in range(3):
+        base = torch.zeros((len(e), 4), dtype=torch.int32, device="cuda")
+        src = torch.from_numpy(e.astype(np.int32)).cuda()
+        base[:, 0] = src[:, 0] * 3 + 7   # some device work the build must wait for ...
+        base[:, 2] = src[:, 1] + 11
+        base[:, 0] = (base[:, 0] - 7) // 3
+        base[:, 2] -= 11
+        t = base[:, 0::2]                  # ... and a non-contiguous view (load() copies it)
+        assert not t.is_contiguous()
+        g = gmbe.load(nu, nv, t)
+        try:
+            r = g.enumerate()
+            assert (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16)), rep
+        finally:
+            g.free()
+
+
+# ---------------------------------------------------------------- real multi-GPU (>= 2 devices)
+def _multi_gpu_worker(rank, world, port, name, mode, q):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_panhlzwc23_b200 as m
+    from paper_conf_sc_panhlzwc23_b200 import dist as gdist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(rank)
+    dev = torch.device("cuda", rank)
+    dist.init_process_group("nccl", rank=rank, world_size=world, device_id=dev)
+    try:
+        nu, nv, e = make_config(name)
+        g = m.load(nu, nv, torch.from_numpy(e.astype(np.int32)).to(dev), device=rank)
+        outs = []
+        if mode == "dynamic":
+            dr = gdist.DynamicRoots(rank, world, device=rank, dev=dev)
+            for _ in range(3):
+                r, tot = dr.enumerate(g)
+                outs.append((r.count, tot["count"], tot["checksum"], tot["nodes"]))
+            q.put((rank, dr.dynamic, dr.error, outs))
+            if rank:
+                dr.close()
+            dist.barrier()
+            if not rank:
+                dr.close()
+        else:
+            for pm in ("interleave", "cost"):
+                r = g.enumerate(part=(rank, world), part_mode=pm)
+                tot = gdist.allreduce_result(r, device=dev)
+                outs.append((r.count, tot["count"], tot["checksum"], tot["nodes"]))
+            q.put((rank, True, None, outs))
+        g.free()
+    except Exception as ex:
+        q.put((rank, False, "%s: %s" % (type(ex).__name__, ex), []))
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("mode", ["dynamic", "static"])
+def test_multi_gpu_distinct_devices(gmbe, mode):
+    """bench.py's N>1 launch on DISTINCT devices (one process per GPU, NCCL): the N1 shared cursor in
+    rank 0's HBM mapped by peers over NVLink (cudaIpcMemLazyEnablePeerAccess, atomicAdd_system
+    across devices), and the static interleave / cost parts -- totals bit-exact vs the golden.
+    Needs >= 2 GPUs (skipped on the one-GPU box)."""
+    import socket
+    import torch
+    import torch.multiprocessing as mp
+    n = torch.cuda.device_count()
+    if n < 2:
+        pytest.skip("needs >= 2 GPUs (found %d)" % n)
+    world = min(n, 8)
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    gd = _gold_cfg()["gh_work"]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_multi_gpu_worker, args=(r, world, port, "gh_work", mode, q)) for r in range(world)]
+    for p in ps:
+        p.start()
+    out = sorted(q.get(timeout=600) for _ in range(world))
+    for p in ps:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    for rank, ok, err, outs in out:
+        assert ok, err
+        for mine, cnt, cks, nodes in outs:
+            assert (cnt, cks, nodes) == (gd["count"], int(gd["checksum"], 16), gd["nodes"])
+    for step in range(len(out[0][3])):
+        assert sum(o[3][step][0] for o in out) == gd["count"]
+
+
+# ---------------------------------------------------------------- N3: GMBE-WARP / GMBE-BLOCK schedulers
+@pytest.mark.parametrize("sched", ["warp", "block"])
+def test_scheduler_variants_small(gmbe, dense_case, sched):
+    """The paper's warp-centric and block-centric schemes (Sec 4.3; the variants of Sec 6.3)
+    walk the same canonical tree as GMBE: identical sets, counts, checksums and counters -- on the
+    paper's G0, ER40, random tiny graphs, the dense block case (deep subtrees) with the Γ-index
+    roots, suffix-mode roots (no Γ index: binary-search maximality), dense-table roots, wide
+    universes (Γ columns), prune off, and output records."""
+    nu, nv, e = g0_edges()
+    for order in ("identity", "degree"):
+        for prune in (True, False):
+            r = _run(gmbe, nu, nv, e, order=order, prune=prune, records=True, scheduler=sched)
+            o = oracle.oracle_mbe(nu, nv, e, order=order, prune=prune, records=True)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques)
+    nu, nv, e = make_config("er40")
+    r = _run(gmbe, nu, nv, e, records=True, scheduler=sched)
+    o = oracle.oracle_mbe(nu, nv, e, records=True)
+    _same(r, o)
+    assert r.bicliques == sorted(o.bicliques)
+    rng = np.random.default_rng(404)
+    for _ in range(60):
+        nu, nv, e = _rand_graph(rng, nmax=14)
+        prune = bool(rng.random() < 0.8)
+        r = _run(gmbe, nu, nv, e, prune=prune, records=True, scheduler=sched)
+        o = oracle.oracle_mbe(nu, nv, e, prune=prune, records=True)
+        _same(r, o)
+        assert r.bicliques == sorted(o.bicliques)
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        for kw in (dict(), dict(debug=128), dict(debug=512), dict(warps_per_sm=16)):
+            r = g.enumerate(records=True, scheduler=sched, **kw)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques), kw
+            assert r.splits == 0 and r.tasks == 0 and r.donations == 0
+        o2 = oracle.oracle_mbe(nu, nv, e, prune=False)
+        _same(g.enumerate(prune=False, scheduler=sched), o2)
+    finally:
+        g.free()
+    for it in range(6):  # wide universes: Γ columns / binary searches
+        nu, nv = int(rng.integers(120, 260)), int(rng.integers(20, 45))
+        e = np.argwhere(rng.random((nu, nv)) < float(rng.uniform(0.25, 0.5))).astype(np.uint32)
+        o = oracle.oracle_mbe(nu, nv, e)
+        for dbg in (0, 128):
+            _same(_run(gmbe, nu, nv, e, debug=dbg, scheduler=sched), o)
+
+
+@pytest.mark.parametrize("name", ["gh", "gh_work", "bx"])
+@pytest.mark.parametrize("sched", ["warp", "block"])
+def test_scheduler_variants_full_config(gmbe, name, sched):
+    gd = _gold_cfg()[name]
+    nu, nv, e = make_config(name)
+    g = gmbe.load(nu, nv, e)
+    try:
+        r = g.enumerate(scheduler=sched)
+        assert (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16))
+        assert (r.nodes, r.nonmax, r.roots_run) == (gd["nodes"], gd["nonmax"], gd["roots_run"])
+        assert r.algo_bytes_cand == gd["algo_bytes_cand"]
+    finally:
+        g.free()

@@ -224,3 +224,16 @@ def test_survey_counter_table():
         assert got == {k: row[k] for k in got}, row
     nu, nv, e = crown_edges(4)
     assert oracle.oracle_mbe(nu, nv, e).checksum == int(kn["crown4"]["checksum"], 16)
+
+
+def test_config_goldens_match_survey_probe():
+    """The stored oracle goldens of the degree-shaped configs reproduce the survey's independent
+    probe numbers (seed-0 Chung-Lu, a third implementation): count, nodes and
+    nonmax of the canonical tree.  Pins the goldens bench.py and the GPU tests compare against."""
+    probe = _gold("survey_known_answers.json")["probe_counts_seed0"]
+    cfg = _gold("configs_oracle.json")
+    for name in ("yg", "gh", "bx", "dblp"):
+        assert cfg[name]["count"] == probe[name], name
+        for k in ("nodes", "nonmax"):
+            if "%s_%s" % (name, k) in probe:
+                assert cfg[name][k] == probe["%s_%s" % (name, k)], (name, k)
