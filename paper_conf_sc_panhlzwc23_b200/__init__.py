@@ -58,7 +58,7 @@ class Opts(ctypes.Structure):
                 ("arena_words", _u64),
                 ("pool_words", _u64), ("queue_cap", _u64), ("cuda_stream", _vp),
                 ("split_wide", _u32), ("thr_min", _u32), ("root_cursor", _vp),
-                ("part_mode", _u32), ("reserved2", _u32)]
+                ("part_mode", _u32), ("root_chunk", _u32)]
 
 
 class CResult(ctypes.Structure):
@@ -176,7 +176,7 @@ class Graph:
     def enumerate(self, prune=True, split=True, bound_height=0, bound_size=0, warps_per_sm=0,
                   part=(0, 1), records=False, rec_cap=1 << 16, ids_cap=1 << 22,
                   per_root=False, root_cycles=False, phases=False, timeline=0, debug=0, thr_min=0, split_wide=0, arena_words=0, pool_words=0, queue_cap=0, stream=None,
-                  root_cursor=None, part_mode="interleave", scheduler="task"):
+                  root_cursor=None, part_mode="interleave", scheduler="task", root_chunk=0):
         """gmbe_enumerate.  records=True allocates device output buffers (torch) and decodes them.
         root_cursor: device address (int) of a shared root-cursor slot (SharedCursor.slot_ptr).
         part_mode: how `part` splits the roots -- "interleave" (degree rank mod N) or "cost" (N4).
@@ -194,6 +194,7 @@ class Graph:
         o.root_cursor = root_cursor
         o.part_mode = PART_MODE[part_mode]
         o.scheduler = SCHEDULER[scheduler]
+        o.root_chunk = root_chunk
         bufs = None
         if records:
             import torch

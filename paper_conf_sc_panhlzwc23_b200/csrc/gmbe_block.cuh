@@ -204,12 +204,12 @@ __device__ int blk_gen_child(const Params& P, const TaskCtx& T, uint32_t* par, u
   later_k = blk_sum64(later_k, S);
   const unsigned long long sra = blk_sum64(sr_abs, S);
   const uint32_t rlen = par[5] + 1 + r_abs;
-  if (tid == 0) {
-    A.nodes++;
-    A.abytes += 4ull * (lc + later_k);
+  if (tid < 32) {  // (warp 0 holds the block's counters, one per lane)
+    A.add(kAcNodes, 1);
+    A.add(kAcAbytes, 4ull * (lc + later_k));
   }
   if (!blk_gamma_is_r(P, T, lpm, lc, rlen, S)) {
-    if (tid == 0) A.nonmax++;
+    if (tid < 32) A.add(kAcNonmax, 1);
     return 0;
   }
   // Output(L', R') (Alg 2 L15)
@@ -219,9 +219,11 @@ __device__ int blk_gen_child(const Params& P, const TaskCtx& T, uint32_t* par, u
   sl = blk_sum64(sl, S);
   const unsigned long long par_sr = ((unsigned long long)par[7] << 32) | par[6];
   const unsigned long long sr = par_sr + P.g.hv[vid] + sra;
+  if (tid < 32) {
+    A.add(kAcCount, 1);
+    A.add(kAcChecksum, pair_hash(P, sl, sr));
+  }
   if (tid == 0) {
-    A.count++;
-    A.checksum += pair_hash(P, sl, sr);
     if (P.per_root) atomicAdd(P.per_root + T.root, 1ull);
     if (T.rlist) T.rlist[par[5]] = vid;
   }
@@ -316,13 +318,14 @@ __global__ void __launch_bounds__(kBlkThreads, 1) k_enum_block(const Params P) {
     const uint32_t rk = S.bc[0];
     __syncthreads();
     if (rk == kNone) break;
-    const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
+    const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = tid < 32 ? A.get(kAcNodes) : 0;
     const long long c0 = P.per_root_cycles ? clock64() : 0;
     if (tid < 32) {  // Alg 3: the root node, built by warp 0 with k_enum's code
       TaskCtx Tc;
       uint32_t* top = nullptr;
       uint32_t* lo = M.dyn;
-      const bool has = run_root(P, rk, M, A, Tc, &top, &lo);
+      const uint32_t lb = P.g.off_v[rk];
+      const bool has = run_root(P, rk, lb, P.g.off_v[rk + 1] - lb, M, A, Tc, &top, &lo);
       if (lane == 0) {
         S.T = Tc;
         S.top = has ? top : nullptr;
@@ -336,19 +339,12 @@ __global__ void __launch_bounds__(kBlkThreads, 1) k_enum_block(const Params P) {
       blk_run_task(P, T, S.top, S.lo, M.dyn_end, A, S);
     }
     __syncthreads();
+    const unsigned long long nn = tid < 32 ? A.get(kAcNodes) - n0 : 0;
     if (tid == 0) {
       if (P.timeline)
-        timeline_rec(P, 0, rk, g0, tl_info(A.nodes - n0, P.g.off_v[rk + 1] - P.g.off_v[rk], 0));
+        timeline_rec(P, 0, rk, g0, tl_info(nn, P.g.off_v[rk + 1] - P.g.off_v[rk], 0));
       if (P.per_root_cycles) atomicAdd(P.per_root_cycles + rk, (unsigned long long)(clock64() - c0));
     }
   }
-  if (tid == 0) {
-    Ctrl* c = P.ctrl;
-    atomicAdd(&c->count, A.count);
-    atomicAdd(&c->checksum, A.checksum);
-    atomicAdd(&c->roots_run, A.roots_run);
-    atomicAdd(&c->nodes, A.nodes);
-    atomicAdd(&c->nonmax, A.nonmax);
-    atomicAdd(&c->abytes, A.abytes);
-  }
+  if (tid < kAcN) atomicAdd(&P.ctrl->count + tid, A.v);  // warp 0: one counter per lane
 }

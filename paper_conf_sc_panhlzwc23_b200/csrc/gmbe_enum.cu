@@ -94,13 +94,28 @@ struct Params {
   uint32_t donate;  // dynamic donation to idle warps (donate_reg)
   uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.thr_min)
   uint32_t split_wide;   // wide-universe split threshold on |C|·⌈|L|/32⌉ (opts.split_wide)
+  uint32_t chunk, chunk_from;  // root claims: `chunk` issue positions per atomic past position chunk_from
   unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1, info]*
   uint64_t timeline_cap;
   unsigned long long* shared_cursor;  // N1: root cursor shared across GPUs / processes (opts.root_cursor)
 };
 
+// Per-warp result counters, one per lane (lane k holds counter k, in Ctrl's field order): a warp-uniform
+// update is one predicated add, and the nine counters cost one register pair instead of nine.
+enum : uint32_t { kAcCount, kAcChecksum, kAcRootsRun, kAcNodes, kAcNonmax, kAcAbytes, kAcSplits, kAcTasks,
+                  kAcDonations, kAcN };
 struct Acc {
-  unsigned long long count, checksum, roots_run, nodes, nonmax, abytes, splits, tasks, donations;
+  unsigned long long v;
+  // add the warp-uniform value x to counter k (called by every lane of the warp)
+  __device__ __forceinline__ void add(uint32_t k, unsigned long long x) {
+    uint32_t l;
+    asm("mov.u32 %0, %%laneid;" : "=r"(l));
+    if (l == k) v += x;
+  }
+  __device__ __forceinline__ unsigned long long get(uint32_t k) const {
+    const uint32_t lo = __shfl_sync(0xffffffffu, (uint32_t)v, k), hi = __shfl_sync(0xffffffffu, (uint32_t)(v >> 32), k);
+    return ((unsigned long long)hi << 32) | lo;
+  }
 #ifdef GMBE_PROFILE
   unsigned long long ph[16];  // profiling build only: SM cycles per phase (opts.phase_cycles)
   long long t0;
@@ -213,10 +228,9 @@ __device__ __forceinline__ unsigned long long warp_sum64r(unsigned long long x) 
   const uint32_t c = __reduce_add_sync(GMBE_FULL, (uint32_t)(x >> 42));
   return (unsigned long long)a + ((unsigned long long)b << 21) + ((unsigned long long)c << 42);
 }
-template <int LPE>
-__device__ __forceinline__ uint32_t group_sum(uint32_t x) {
-#pragma unroll
-  for (int o = LPE / 2; o; o >>= 1) x += __shfl_xor_sync(GMBE_FULL, x, o);
+// sum over aligned groups of lpe lanes (lpe a power of two <= 32; runtime, one code copy)
+__device__ __forceinline__ uint32_t group_sum(uint32_t x, uint32_t lpe) {
+  for (uint32_t o = lpe >> 1; o; o >>= 1) x += __shfl_xor_sync(GMBE_FULL, x, o);
   return x;
 }
 __device__ __forceinline__ uint32_t next_pow2(uint32_t x) { return x <= 1 ? 1u : 1u << (32 - __clz(x - 1)); }
@@ -538,7 +552,7 @@ __device__ bool task_publish(const Params& P, const TaskCtx& T, uint32_t lmap, u
     s[node_off + 3] = 0;      // next candidate
     s[node_off + 4] = kNone;  // no parent: top of its task
   }
-  A.tasks++;
+  A.add(kAcTasks, 1);
   __threadfence();  // release the task before it becomes visible in the queue
   __syncwarp();
   if (lane == 0) queue_push(P, off16);
@@ -792,10 +806,10 @@ __device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_cols_is_r(const TaskCtx& T, cons
 // candidates are compacted in place (Thm 4.1 prunes removed), so par[0] shrinks.
 // Returns 0: non-maximal; 1: maximal leaf (C' empty); 2: maximal with C' != ∅ (ch holds the child
 // node record, header filled except the parent link).
-template <int LPE>
+// LPE (lanes per candidate entry, 4..32) is a runtime value: one code copy serves every width
 __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint32_t i, uint32_t* ch, Acc& A,
-                         unsigned long long* smem) {
-  constexpr uint32_t G = 32 / LPE;
+                         unsigned long long* smem, const uint32_t LPE) {
+  const uint32_t G = 32 / LPE;
   const uint32_t lane = lane_id(), sub = lane & (LPE - 1), grp = lane / LPE;
   const bool leader = sub == 0;
   const uint32_t W = T.W, E = T.E;
@@ -837,7 +851,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
       id = ej[W];
       kp = ej[W + 1];
     }
-    cnt = group_sum<LPE>(cnt);
+    cnt = group_sum(cnt, LPE);
     const bool pruned = in && P.prune && cnt == kp;
     const bool surv = in && !pruned;
     const bool absorb = in && cnt == lc;
@@ -877,8 +891,8 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
     __syncwarp();
   }
   if (lane == 0) par[0] = i + 1 + nsurv;
-  A.nodes++;
-  A.abytes += 4ull * (lc + warp_sum64(later_k));
+  A.add(kAcNodes, 1);
+  A.add(kAcAbytes, 4ull * (lc + warp_sum64(later_k)));
   const uint32_t rlen = par[5] + 1 + r_abs;
   __syncwarp();
   unsigned long long* gscr = (unsigned long long*)align4(cent + (size_t)nCc * E);
@@ -899,7 +913,7 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
 #endif
   PH_STOP(A, 5);
   if (!maximal) {
-    A.nonmax++;
+    A.add(kAcNonmax, 1);
     return 0;
   }
   // Output(L', R') (Alg 2 L15)
@@ -909,8 +923,8 @@ __device__ int gen_child(const Params& P, const TaskCtx& T, uint32_t* par, uint3
   for (uint32_t w = lane; w < W; w += 32)
     for (uint32_t word = lpm[w]; word; word &= word - 1) sl += hash_u(P, T.map[w * 32 + __ffs(word) - 1]);
   sl = warp_sum64(sl);
-  A.count++;
-  A.checksum += pair_hash(P, sl, sr);
+  A.add(kAcCount, 1);
+  A.add(kAcChecksum, pair_hash(P, sl, sr));
   if (P.per_root && lane == 0) atomicAdd(P.per_root + T.root, 1ull);
   if (T.rlist) {
     if (lane == 0) T.rlist[par[5]] = vid;
@@ -1058,8 +1072,8 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
     __syncwarp();
   }
   if (lane == 0) par[0] = i + 1 + nsurv;
-  A.nodes++;
-  A.abytes += 4ull * (lc + warp_sum64r(later_k));
+  A.add(kAcNodes, 1);
+  A.add(kAcAbytes, 4ull * (lc + warp_sum64r(later_k)));
   const uint32_t rlen = par[5] + 1 + r_abs;
   PH_STOP(A, 4);
   bool maximal;
@@ -1076,7 +1090,7 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
   }
   PH_STOP(A, 5);
   if (!maximal) {
-    A.nonmax++;
+    A.add(kAcNonmax, 1);
     return 0;
   }
   // Output(L', R') (Alg 2 L15)
@@ -1084,8 +1098,8 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
   const unsigned long long sl =
       warp_sum64r(((lm >> lane) & 1ull ? T.hu0 : 0ull) + ((lm >> (lane + 32)) & 1ull ? T.hu1 : 0ull));
   const unsigned long long sr = par_sr + P.g.hv[vid] + warp_sum64r(sr_abs);
-  A.count++;
-  A.checksum += pair_hash(P, sl, sr);
+  A.add(kAcCount, 1);
+  A.add(kAcChecksum, pair_hash(P, sl, sr));
   if (P.per_root && lane == 0) atomicAdd(P.per_root + T.root, 1ull);
   if (T.rlist) {
     if (lane == 0) T.rlist[par[5]] = vid;
@@ -1224,7 +1238,7 @@ __device__ GMBE_DONATE_ATTR bool donate_reg(const Params& P, const TaskCtx& T, u
   if (!task_publish(P, T, lmap, T.rlist ? rk : 0, scratch, words, A)) return false;
   if (lane == 0) st[k].next = 32;  // the donated children are no longer this warp's
   __syncwarp();
-  A.donations++;
+  A.add(kAcDonations, 1);
   return true;
 }
 
@@ -1262,6 +1276,7 @@ __device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& 
       C = st[d].C;
       next = st[d].next;
       rlen = st[d].rlen;
+      __syncwarp();  // every lane has read level d before lane 0 overwrites it at the next push
       continue;
     }
     const uint32_t i = __ffs(avail) - 1;
@@ -1275,8 +1290,8 @@ __device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& 
     const uint32_t ab = __ballot_sync(GMBE_FULL, inl && kc == lc);
     const uint32_t cd = __ballot_sync(GMBE_FULL, inl && kc > 0 && kc < lc);
     C &= ~pr;  // Thm 4.1
-    A.nodes++;
-    A.abytes += 4ull * (lc + __reduce_add_sync(GMBE_FULL, inl ? kp : 0u));
+    A.add(kAcNodes, 1);
+    A.add(kAcAbytes, 4ull * (lc + __reduce_add_sync(GMBE_FULL, inl ? kp : 0u)));
     const uint32_t rl = rlen + 1 + __popc(ab);
     bool maximal;
     if (lc == 1) {
@@ -1293,7 +1308,7 @@ __device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& 
       maximal = gamma_is_r(P, scratch, T.W, T.map, lc, rl, (unsigned long long*)(scratch + 4), nullptr);
     }
     if (!maximal) {
-      A.nonmax++;
+      A.add(kAcNonmax, 1);
       continue;
     }
     // Output(L', R') (Alg 2 L15)
@@ -1301,8 +1316,8 @@ __device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& 
     const unsigned long long srn = SR + shfl64(hvj, i) + warp_sum64r(((ab >> lane) & 1u) ? hvj : 0ull);
     const unsigned long long sl =
         warp_sum64r(((lp >> lane) & 1ull ? T.hu0 : 0ull) + ((lp >> (lane + 32)) & 1ull ? T.hu1 : 0ull));
-    A.count++;
-    A.checksum += pair_hash(P, sl, srn);
+    A.add(kAcCount, 1);
+    A.add(kAcChecksum, pair_hash(P, sl, srn));
     if (P.per_root && lane == 0) atomicAdd(P.per_root + T.root, 1ull);
     if (T.rlist) {
       if (lane == 0) T.rlist[rlen] = idi;
@@ -1385,9 +1400,13 @@ struct ThrSmem {
   uint32_t deg[64];            // degree of each universe vertex
   uint32_t id[32];             // rank of each candidate
 };
+// One stacked DFS level of a lane (16 B): the node's L, candidate mask C and R-mask Rm.  Its SR and
+// `next` are not stored: the child above it has Rm' = Rm ∪ {i} ∪ absorbed with every absorbed
+// candidate ranked after the branch candidate i, so next = i + 1 = ffs(Rm' \ Rm) and
+// SR = SR' - Σ_{c ∈ Rm' \ Rm} hV(c) (derived on pop, and for donation from the current node).
 struct ThrLevel {
-  unsigned long long L, SR;
-  uint32_t C, Rm, next, pad;
+  unsigned long long L;
+  uint32_t C, Rm;
 };
 
 // one output record from one lane: L' = bits of lp over map, R' = the job's R list + candidates rm
@@ -1450,7 +1469,7 @@ __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const
   }
   __syncwarp();
   if (!task_publish(P, T, lmap, T.rlist ? rk : 0, scratch, words, A)) return false;
-  A.donations++;
+  A.add(kAcDonations, 1);
   return true;
 }
 
@@ -1465,6 +1484,9 @@ __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const
 #endif
 #ifndef GMBE_THR_DONATE_MASK
 #define GMBE_THR_DONATE_MASK 3  // run_thr checks ctrl.hungry every (mask + 1) steps
+#endif
+#ifndef GMBE_ROOT_CHUNK
+#define GMBE_ROOT_CHUNK 16  // light roots claimed per atomic (opts.root_chunk)
 #endif
 #ifndef GMBE_THR_MIN_EST
 #define GMBE_THR_MIN_EST 16  // jobs with fewer adjacency bits (Σ(k-1)) stay on run_reg (setup > work)
@@ -1610,11 +1632,12 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
           break;
         }
         d--;
+        const uint32_t rmp = stk[d].Rm, diff = Rm & ~rmp;  // {i} ∪ absorbed of the finished child
+        next = __ffs(diff);
+        for (uint32_t m = diff; m; m &= m - 1) SR -= ts->hv[__ffs(m) - 1];
         L = stk[d].L;
-        SR = stk[d].SR;
         C = stk[d].C;
-        Rm = stk[d].Rm;
-        next = stk[d].next;
+        Rm = rmp;
         dmask &= ~(1u << d);
       }
     }
@@ -1638,14 +1661,15 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
         uint32_t kC = 0, kRm = 0, knext = 0;
         if (lane == src) {
           kL = stk[k].L;
-          kSR = stk[k].SR;
           kC = stk[k].C;
           kRm = stk[k].Rm;
-          knext = stk[k].next;
+          knext = __ffs((k + 1 < d ? stk[k + 1].Rm : Rm) & ~kRm);
+          kSR = SR;
+          for (uint32_t m = Rm & ~kRm; m; m &= m - 1) kSR -= ts->hv[__ffs(m) - 1];
         }
         if (donate_thr(P, T, lmap, A, ts, nC, rlen0, src, kL, kSR, kC, kRm, knext, scratch, scratch_end) &&
             lane == src) {
-          stk[k].next = 32;
+          stk[k].C &= knext >= 32 ? GMBE_FULL : (1u << knext) - 1u;  // its remaining children left
           dmask &= ~(1u << k);
         }
       }
@@ -1660,11 +1684,16 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
         if (dmask && rd < nd) {
           const uint32_t k = __ffs(dmask) - 1;
           unsigned long long* o = slot + 4 * rd;
+          const uint32_t rmk = stk[k].Rm, ck = stk[k].C;
+          const uint32_t nk = __ffs((k + 1 < d ? stk[k + 1].Rm : Rm) & ~rmk);
+          unsigned long long srk = SR;
+          for (uint32_t m = Rm & ~rmk; m; m &= m - 1) srk -= ts->hv[__ffs(m) - 1];
           o[0] = stk[k].L;
-          o[1] = stk[k].SR;
-          o[2] = ((unsigned long long)stk[k].Rm << 32) | stk[k].C;
-          o[3] = ((unsigned long long)(bd + k) << 32) | stk[k].next;
-          stk[k].next = 32;  // the remaining children of level k are no longer this lane's
+          o[1] = srk;
+          o[2] = ((unsigned long long)rmk << 32) | ck;
+          o[3] = ((unsigned long long)(bd + k) << 32) | nk;
+          // the remaining children of level k are no longer this lane's
+          stk[k].C = ck & (nk >= 32 ? GMBE_FULL : (1u << nk) - 1u);
           dmask &= ~(1u << k);
         }
         __syncwarp();
@@ -1760,10 +1789,8 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
 #endif
     // push (Alg 2 L16)
     stk[d].L = L;
-    stk[d].SR = SR;
     stk[d].C = C;
     stk[d].Rm = Rm;
-    stk[d].next = next;
     if (next < 32 && (C & (GMBE_FULL << next))) dmask |= 1u << d;
     d++;
     L = lp;
@@ -1786,43 +1813,45 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     }
   }
 #endif
-  A.nodes += warp_sum(n_nodes);
-  A.nonmax += warp_sum(n_nonmax);
-  A.count += warp_sum(n_count);
-  A.abytes += 4ull * warp_sum64r(abytes);
-  A.checksum += warp_sum64r(cks);
+  A.add(kAcNodes, warp_sum(n_nodes));
+  A.add(kAcNonmax, warp_sum(n_nonmax));
+  A.add(kAcCount, warp_sum(n_count));
+  A.add(kAcAbytes, 4ull * warp_sum64r(abytes));
+  A.add(kAcChecksum, warp_sum64r(cks));
   PH_STOP(A, 4);
   return true;
 }
 
-template <int LPE>
+// SMALL: universes <= 64 bits (16-byte entries, register / thread tiers); else wide universes with
+// lpe lanes per candidate entry
+template <bool SMALL>
 __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint32_t* stack_lo, uint32_t* stack_hi,
-                         uint32_t lmap, Acc& A, unsigned long long* smem, ThrSmem* ts) {
+                         uint32_t lmap, Acc& A, unsigned long long* smem, ThrSmem* ts, uint32_t lpe) {
   const uint32_t lane = lane_id();
   uint32_t* cur = top;
   uint32_t* sp = stack_lo;  // first free word
   const bool split_mode = heavy(P, top[2], top[0]) || late_heavy(P, top[2], top[0]);
-  if (split_mode) A.splits++;
+  if (split_mode) A.add(kAcSplits, 1);
   // register-resident DFS (one inline site): the whole task if its top has <= 32 candidates,
   // else every pushed child with <= 32 candidates
   const uint32_t* reg = nullptr;
   uint32_t* reg_scratch = stack_lo;
-  if constexpr (LPE == 0) {
+  if constexpr (SMALL) {
     if (top[0] <= 32) reg = top;
   }
   while (true) {
-    if constexpr (LPE == 0) {
+    if constexpr (SMALL) {
       if (reg) {
         const bool st = split_mode && reg == top;  // heavy top: publish its children (run_reg)
 #ifndef GMBE_PROFILE
-        const unsigned long long n0 = A.nodes;
+        const unsigned long long n0 = A.get(kAcNodes);
 #endif
         const bool thr = !st && !(P.debug & 16) && run_thr(P, T, reg, lmap, A, ts, smem, reg_scratch, stack_hi);
         if (!thr) run_reg(P, T, reg, lmap, A, (RegLevel*)smem, reg_scratch, stack_hi, st, smem);
 #ifndef GMBE_PROFILE
         if ((P.debug & 32) && lane == 0) {  // path statistics (experiments): jobs / nodes per tier
           atomicAdd(&P.ctrl->phase[thr ? 0 : 2], 1ull);
-          atomicAdd(&P.ctrl->phase[thr ? 1 : 3], A.nodes - n0);
+          atomicAdd(&P.ctrl->phase[thr ? 1 : 3], A.get(kAcNodes) - n0);
         }
 #endif
         if (reg == top) return;
@@ -1846,17 +1875,17 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     if (!fits(P, sp + need, stack_hi)) return;
     uint32_t* ch = sp;  // children are generated on this warp's stack; only a published one is copied
     int r;
-    if constexpr (LPE == 0) r = gen_child_small(P, T, cur, i, ch, A, smem);
-    else r = gen_child<LPE>(P, T, cur, i, ch, A, smem);
+    if constexpr (SMALL) r = gen_child_small(P, T, cur, i, ch, A, smem);
+    else r = gen_child(P, T, cur, i, ch, A, smem, lpe);
     // Alg 4 L25: hand the child to the task queue as a self-contained subtask -- every child of a
     // heavy top, and (wide universes) any child that is itself heavy (reading B4)
-    if (r == 2 && ((split_mode && cur == top) || (LPE != 0 && heavy_wide(P, lmap, ch[0])))) {
+    if (r == 2 && ((split_mode && cur == top) || (!SMALL && heavy_wide(P, lmap, ch[0])))) {
       PH_START(A);
       const bool done = task_publish(P, T, lmap, T.rlist ? ch[5] : 0, ch, rec_words(T, ch), A);
       PH_STOP(A, 7);
       if (done) continue;
     }
-    if constexpr (LPE == 0) {
+    if constexpr (SMALL) {
       if (r == 2 && ch[0] <= 32) {  // the child's subtree fits the register-resident DFS
         reg = ch;
         reg_scratch = align4(ch + rec_words(T, ch));
@@ -1879,12 +1908,10 @@ __device__ GMBE_NI_IF(GMBE_NI_DISPATCH) void dispatch_task(const Params& P, Task
                               uint32_t lmap, Acc& A, unsigned long long* smem, ThrSmem* ts) {
   if (T.W <= 2) {
     small_task_init(P, T, lmap);
-    run_task<0>(P, T, top, lo, hi, lmap, A, smem, ts);
+    run_task<true>(P, T, top, lo, hi, lmap, A, smem, ts, 0);
+  } else {  // lanes per entry: the row words rounded up to a power of two, 4..32
+    run_task<false>(P, T, top, lo, hi, lmap, A, smem, ts, T.W <= 4 ? 4u : T.W <= 8 ? 8u : T.W <= 16 ? 16u : 32u);
   }
-  else if (T.W <= 4) run_task<4>(P, T, top, lo, hi, lmap, A, smem, ts);  // W > 2 from here
-  else if (T.W <= 8) run_task<8>(P, T, top, lo, hi, lmap, A, smem, ts);
-  else if (T.W <= 16) run_task<16>(P, T, top, lo, hi, lmap, A, smem, ts);
-  else run_task<32>(P, T, top, lo, hi, lmap, A, smem, ts);
 }
 
 // ---------------------------------------------------------------- root task (a3)
@@ -1938,11 +1965,10 @@ __device__ bool earlier_dominator(const DevGraph& g, const uint32_t* Lr, uint32_
 // Root v_s (rank r): L_r = N(v_s); wedge scan of N2(v_s) with k(v) = |N(v) ∩ L_r|.  Emits the root
 // biclique and, if it has candidates, prepares its node record as a task (Tc, *top, stack from *lo)
 // for the caller's single dispatch site; returns whether it did.
-__device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, WarpMem& M, Acc& A, TaskCtx& Tc,
-                                                  uint32_t** top, uint32_t** lo) {
+__device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, uint32_t lb, uint32_t l, WarpMem& M,
+                                                  Acc& A, TaskCtx& Tc, uint32_t** top, uint32_t** lo) {
   const uint32_t lane = lane_id();
-  const DevGraph& g = P.g;
-  const uint32_t lb = g.off_v[r], l = g.off_v[r + 1] - lb;
+  const DevGraph& g = P.g;  // N(v_s) = adj_v[lb, lb + l) (prefetched by the caller)
   if (l == 0) return false;  // isolated vertex: in no biclique (A17)
   const uint32_t* Lr = g.adj_v + lb;
   const unsigned long long hv_r = g.hv[r];  // issued early, consumed at the root's emission
@@ -1952,7 +1978,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
     wp += g.off_u[u + 1] - g.off_u[u];
   }
   const uint32_t wedges = warp_sum(wp);
-  A.abytes += 4ull * (l + wedges);
+  A.add(kAcAbytes, 4ull * (l + wedges));
   // Suffix mode (B200 addition, reading B5): a root with many wedges but few of them to
   // later-ranked vertices (high degree rank: few candidates, huge excluded set) counts k only over
   // the rank suffix of each list; the skip test (Alg 3 L7) then looks for an earlier dominator
@@ -2092,13 +2118,13 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, W
   uint32_t* rec = align4(aux + (want_aux ? aux_words : 0));
   const uint64_t rec_need = kHdr + W4 + (uint64_t)nC * E;
   if (sort_fits && !skip && fits(P, rec + rec_need + 64, M.dyn_end)) {
-    A.roots_run++;
+    A.add(kAcRootsRun, 1);
     sr = warp_sum64r(sr) + hv_r;
     unsigned long long sl = 0;
     for (uint32_t j = lane; j < l; j += 32) sl += hash_u(P, Lr[j]);
     sl = warp_sum64r(sl);
-    A.count++;  // emit (L_r, R_r) (A5)
-    A.checksum += pair_hash(P, sl, sr);
+    A.add(kAcCount, 1);  // emit (L_r, R_r) (A5)
+    A.add(kAcChecksum, pair_hash(P, sl, sr));
     if (P.per_root && lane == 0) atomicAdd(P.per_root + r, 1ull);
     if (M.rbuf) {
       if (lane == 0) M.rbuf[0] = r;
@@ -2361,6 +2387,7 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
   Acc A = {};
   bool roots_done = false, is_hungry = false;
   uint32_t idle = 0;
+  uint32_t ck_pos = 0, ck_end = 0, ck_base = 0, ck_rk = 0, ck_lb = 0, ck_l = 0;  // claimed root chunk
   while (true) {
     // work item: a queued split subtask first (Alg 4 L3-4), else the next root (Alg 4 L6, heaviest =
     // highest rank first); both end in the single dispatch site below
@@ -2369,10 +2396,12 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
     uint32_t* lo = M.dyn;
     uint32_t lmap = 0, kind = 2, item = 0, tl_l = 0, tl_c = 0;
     const long long c0 = P.per_root_cycles ? clock64() : 0;
-    const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.nodes;
+    const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.get(kAcNodes);
     uint32_t task = kNone;
-    if (lane == 0) task = queue_pop(P);
+    // the queue is polled between root chunks (inside a chunk of light roots the warp keeps going)
+    if (lane == 0 && ck_pos == ck_end) task = queue_pop(P);
     task = __shfl_sync(GMBE_FULL, task, 0);
+    bool release = true;  // this item ends a unit of `pending` (a task, or a chunk's last root)
     if (task != kNone) {
       if (is_hungry) {
         if (lane == 0) atomicAdd(&P.ctrl->hungry.v, ~0ull);
@@ -2403,32 +2432,53 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
       tl_l = top[2];
       tl_c = top[0];
     } else if (!roots_done) {
-      unsigned long long t = 0;
-      if (lane == 0) {
-        atomicAdd(&P.ctrl->pending.v, 1ull);
-        // N1: a cursor shared by every GPU takes a system-scope atomic over NVLink
-        t = P.shared_cursor ? atomicAdd_system(P.shared_cursor, 1ull) : atomicAdd(&P.ctrl->root_cursor.v, 1ull);
+      if (ck_pos == ck_end) {
+        // claim a chunk of consecutive issue positions with ONE atomic: single roots in the heavy
+        // head of the issue list, P.chunk roots once this warp has seen positions past
+        // P.chunk_from (the estimate may be stale; any K gives disjoint ranges)
+        const uint32_t K = ck_end >= P.chunk_from ? P.chunk : 1u;
+        unsigned long long t = 0;
+        if (lane == 0) {
+          atomicAdd(&P.ctrl->pending.v, 1ull);
+          // N1: a cursor shared by every GPU takes a system-scope atomic over NVLink
+          t = P.shared_cursor ? atomicAdd_system(P.shared_cursor, (unsigned long long)K)
+                              : atomicAdd(&P.ctrl->root_cursor.v, (unsigned long long)K);
+        }
+        t = __shfl_sync(GMBE_FULL, t, 0);
+        if (t < P.n_roots) {
+          ck_pos = (uint32_t)t;
+          ck_end = (uint32_t)min(t + K, (unsigned long long)P.n_roots);
+          ck_base = ck_pos;
+          // prefetch the chunk: lane j holds the root at position ck_base + j and its N(v) range
+          const uint32_t q = ck_pos + lane;
+          ck_rk = q < ck_end ? P.issue[q] : 0u;
+          ck_lb = q < ck_end ? P.g.off_v[ck_rk] : 0u;
+          ck_l = q < ck_end ? P.g.off_v[ck_rk + 1] - ck_lb : 0u;
+        } else {
+          if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
+          roots_done = true;
+        }
       }
-      t = __shfl_sync(GMBE_FULL, t, 0);
-      if (t < P.n_roots) {
-        const uint32_t rk = P.issue[t];
+      if (!roots_done) {
+        const uint32_t jq = ck_pos - ck_base;
+        const uint32_t rk = __shfl_sync(GMBE_FULL, ck_rk, jq);
+        const uint32_t rlb = __shfl_sync(GMBE_FULL, ck_lb, jq), rl = __shfl_sync(GMBE_FULL, ck_l, jq);
+        ck_pos++;
+        release = ck_pos == ck_end;
         kind = 0;
         item = rk;
-        if (run_root(P, rk, M, A, Tc, &top, &lo)) lmap = top[2];
+        if (run_root(P, rk, rlb, rl, M, A, Tc, &top, &lo)) lmap = top[2];
         if (P.debug & 1024) top = nullptr;  // experiments: root construction only (no subtrees)
-        tl_l = P.timeline ? P.g.off_v[rk + 1] - P.g.off_v[rk] : 0;
-      } else {
-        if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
-        roots_done = true;
+        tl_l = rl;
       }
     }
     if (kind != 2) {
       if (top) dispatch_task(P, Tc, top, lo, M.dyn_end, lmap, A, M.sm_sort, &s_thr[threadIdx.x >> 5]);
-      if (P.timeline) timeline_rec(P, kind, item, g0, tl_info(A.nodes - n0, tl_l, tl_c));
+      if (P.timeline) timeline_rec(P, kind, item, g0, tl_info(A.get(kAcNodes) - n0, tl_l, tl_c));
       if (P.per_root_cycles && lane == 0)
         atomicAdd(P.per_root_cycles + item, (unsigned long long)(clock64() - c0));
       __syncwarp();
-      if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
+      if (lane == 0 && release) atomicAdd(&P.ctrl->pending.v, ~0ull);
       idle = 0;
       continue;
     }
@@ -2445,17 +2495,9 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
     __nanosleep(idle < 4 ? 500 : (idle < 16 ? 2000 : 8000));  // exponential-ish backoff
     idle++;
   }
+  if (lane < kAcN) atomicAdd(&P.ctrl->count + lane, A.v);  // Ctrl's counters, in kAc* order
   if (lane == 0) {
     Ctrl* c = P.ctrl;
-    atomicAdd(&c->count, A.count);
-    atomicAdd(&c->checksum, A.checksum);
-    atomicAdd(&c->roots_run, A.roots_run);
-    atomicAdd(&c->nodes, A.nodes);
-    atomicAdd(&c->nonmax, A.nonmax);
-    atomicAdd(&c->abytes, A.abytes);
-    atomicAdd(&c->splits, A.splits);
-    atomicAdd(&c->tasks, A.tasks);
-    atomicAdd(&c->donations, A.donations);
 #ifdef GMBE_PROFILE
     if (P.profile)
       for (int k = 0; k < 16; k++) atomicAdd(&c->phase[k], A.ph[k]);
@@ -2599,8 +2641,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   }
   const uint32_t parts = o.part_count ? o.part_count : 1;
   if (o.part_index >= parts) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: part_index >= part_count");
-  if (o.part_mode > GMBE_PART_COST || o.reserved2)
-    return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: bad part_mode / reserved2");
+  if (o.part_mode > GMBE_PART_COST) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: bad part_mode");
   if (o.scheduler > GMBE_SCHED_BLOCK) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: bad scheduler");
   if (o.root_cursor && parts > 1)
     return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: root_cursor needs part_count <= 1");
@@ -2806,6 +2847,10 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   P.donate = (o.reserved0 & 4) || o.scheduler != GMBE_SCHED_TASK ? 0 : 1;
   if (o.scheduler == GMBE_SCHED_WARP) P.debug |= 16;  // one warp per node: no thread-level tier
   P.thr_min_est = o.thr_min ? o.thr_min : GMBE_THR_MIN_EST;
+  // root claims: after the heavy head of the issue list (the first 1/8 of the positions, one root
+  // per atomic), a warp claims root_chunk consecutive positions per atomic (default 16, <= 32)
+  P.chunk = o.root_chunk ? std::min<uint32_t>(o.root_chunk, 32u) : GMBE_ROOT_CHUNK;
+  P.chunk_from = P.n_roots / 8;
   P.split_wide = o.split_wide ? o.split_wide : GMBE_SPLIT_WIDE;
   P.timeline = (unsigned long long*)o.timeline;
   P.timeline_cap = o.timeline_cap;

@@ -1,23 +1,26 @@
 // gmbe_graph.cu -- device graph build (DESIGN.md steps a1-a2; Sec 5 "Pre-processing",
 // P:1014-1025, and multi-edge removal).
 //
-//   a1  edge ingest -> validate ids -> orient (V := smaller side) -> pack (u<<32|v)
-//       -> radix sort -> unique (dedupe)
+//   a1  edge ingest -> validate ids -> orient (V := smaller side) -> pack (u<<bv|v)
+//       -> radix sort -> first-copy flags + their scan (dedupe without a host round trip)
 //   a2  degrees -> global vertex order (ascending degree, ties by id)
-//       -> CSR of V by rank (u ascending) and CSR of U (ranks ascending) -> Δ(U), Δ(V), wedge
-//       bound (>= Δ2(V)) -> per-rank checksum hash table.
+//       -> CSR of V by rank (u ascending) and CSR of U (ranks ascending) by two stable partial-key
+//       sorts -> Δ(U), Δ(V), wedge bound (>= Δ2(V)) -> per-rank checksum hash table; one host
+//       synchronisation at the very end.
 // Sorting / scanning / selection use CUB (library primitives); everything else is our kernels.
 #include <cub/cub.cuh>
 
+#include <cstring>
 #include <vector>
 
 #include "gmbe_internal.cuh"
 
 namespace {
 
+// a1: validate, orient and pack one edge per key: (u << bv) | v, bv = bits of the library's V ids
 __global__ void k_pack_edges(const uint32_t* __restrict__ e, uint64_t m, uint32_t n_u, uint32_t n_v,
-                             uint32_t swapped, unsigned long long* __restrict__ keys,
-                             int* __restrict__ bad) {
+                             uint32_t swapped, uint32_t bv, unsigned long long* __restrict__ keys,
+                             uint32_t* __restrict__ bad) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
        i += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t u = e[2 * i], v = e[2 * i + 1];
@@ -31,32 +34,40 @@ __global__ void k_pack_edges(const uint32_t* __restrict__ e, uint64_t m, uint32_
       u = v;
       v = t;
     }
-    keys[i] = ((unsigned long long)u << 32) | v;
+    keys[i] = ((unsigned long long)u << bv) | v;
   }
 }
 
-__global__ void k_degrees(const unsigned long long* __restrict__ keys, uint64_t m,
-                          uint32_t* __restrict__ deg_u, uint32_t* __restrict__ deg_v) {
+// a1 dedupe on the (u, v)-sorted keys: flag[i] = first copy of its edge; degrees of
+// the unique edges (a2)
+__global__ void k_unique_degrees(const unsigned long long* __restrict__ keys, uint64_t m, uint32_t bv,
+                                 uint32_t* __restrict__ flag, uint32_t* __restrict__ deg_u,
+                                 uint32_t* __restrict__ deg_v) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
        i += (uint64_t)gridDim.x * blockDim.x) {
-    unsigned long long k = keys[i];
-    atomicAdd(&deg_u[k >> 32], 1u);
-    atomicAdd(&deg_v[(uint32_t)k], 1u);
+    const unsigned long long k = keys[i];
+    const bool first = i == 0 || keys[i - 1] != k;
+    flag[i] = first;
+    if (first) {
+      atomicAdd(&deg_u[k >> bv], 1u);
+      atomicAdd(&deg_v[(uint32_t)(k & ((1ull << bv) - 1))], 1u);
+    }
   }
 }
 
-__global__ void k_order_keys(const uint32_t* __restrict__ deg_v, uint32_t n_v, uint32_t identity,
+// sort keys of the global vertex order: (deg << bv) | v -- ascending degree, ties by id (A8)
+__global__ void k_order_keys(const uint32_t* __restrict__ deg_v, uint32_t n_v, uint32_t identity, uint32_t bv,
                              unsigned long long* __restrict__ out) {
   for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n_v; v += gridDim.x * blockDim.x)
-    out[v] = identity ? (unsigned long long)v : (((unsigned long long)deg_v[v] << 32) | v);
+    out[v] = identity ? (unsigned long long)v : (((unsigned long long)deg_v[v] << bv) | v);
 }
 
-__global__ void k_rank_maps(const unsigned long long* __restrict__ sorted, uint32_t n_v,
+__global__ void k_rank_maps(const unsigned long long* __restrict__ sorted, uint32_t n_v, uint32_t bv,
                             uint32_t side_v, uint32_t* __restrict__ rank2id,
                             uint32_t* __restrict__ id2rank, const uint32_t* __restrict__ deg_v,
                             uint32_t* __restrict__ deg_by_rank, unsigned long long* __restrict__ hv) {
   for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < n_v; r += gridDim.x * blockDim.x) {
-    uint32_t id = (uint32_t)sorted[r];
+    const uint32_t id = (uint32_t)(sorted[r] & ((1ull << bv) - 1));
     rank2id[r] = id;
     id2rank[id] = r;
     deg_by_rank[r] = deg_v[id];
@@ -64,22 +75,26 @@ __global__ void k_rank_maps(const unsigned long long* __restrict__ sorted, uint3
   }
 }
 
-__global__ void k_rekey(const unsigned long long* __restrict__ keys, uint64_t m,
-                        const uint32_t* __restrict__ id2rank, unsigned long long* __restrict__ kv,
-                        unsigned long long* __restrict__ ku) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
+// unique edges in (u, v) order -> (rank(v), u) pairs at their deduplicated position (the exclusive
+// scan of the flags); positions [m, m0) get the sentinel key n_v, which every later sort keeps last
+__global__ void k_rank_pairs(const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ flag,
+                             const uint32_t* __restrict__ pos, uint64_t m0, uint32_t bv,
+                             const uint32_t* __restrict__ id2rank, uint32_t n_u, uint32_t n_v,
+                             uint32_t* __restrict__ pk, uint32_t* __restrict__ pv, uint32_t* __restrict__ m_out) {
+  const uint32_t m = m0 ? pos[m0 - 1] + flag[m0 - 1] : 0u;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m0;
        i += (uint64_t)gridDim.x * blockDim.x) {
-    unsigned long long k = keys[i];
-    uint32_t u = (uint32_t)(k >> 32), r = id2rank[(uint32_t)k];
-    kv[i] = ((unsigned long long)r << 32) | u;
-    ku[i] = ((unsigned long long)u << 32) | r;
+    if (flag[i]) {
+      const unsigned long long k = keys[i];
+      pk[pos[i]] = id2rank[(uint32_t)(k & ((1ull << bv) - 1))];
+      pv[pos[i]] = (uint32_t)(k >> bv);
+    }
+    if (i >= m) {
+      pk[i] = n_v;
+      pv[i] = n_u;
+    }
+    if (i == 0) *m_out = m;
   }
-}
-
-__global__ void k_low32(const unsigned long long* __restrict__ k, uint64_t m, uint32_t* __restrict__ out) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m;
-       i += (uint64_t)gridDim.x * blockDim.x)
-    out[i] = (uint32_t)k[i];
 }
 
 // one warp per V rank: wedge count Σ_{u∈N(v)} |N(u)| and the maxima.
@@ -88,34 +103,57 @@ __global__ void k_issue(const unsigned long long* __restrict__ keys, uint32_t n,
     issue[i] = ~(uint32_t)keys[i];
 }
 
+// one warp per V rank: wedge count Σ_{u∈N(v)} |N(u)| (the issue key) and the maxima.  The maxima are
+// reduced per block first (one atomic per block and quantity: a per-rank atomic on four addresses
+// serialises millions of atomics on light-root graphs).
 __global__ void k_bounds(const uint32_t* __restrict__ off_v, const uint32_t* __restrict__ adj_v,
                          const uint32_t* __restrict__ off_u, uint32_t n_v, uint32_t n_u,
                          uint32_t* __restrict__ maxes /* [0]=Δ(V) [1]=Δ(U) [2]=wedge bound */,
                          unsigned long long* __restrict__ rec_bound, unsigned long long* __restrict__ cost_key) {
-  uint32_t lane = threadIdx.x & 31;
-  uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  __shared__ unsigned long long red[4][32];
+  const uint32_t lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+  uint32_t mdv = 0, mdu = 0, mw = 0;
+  unsigned long long mrec = 0;
   for (uint32_t r = warp; r < n_v; r += nw) {
-    uint32_t b = off_v[r], e = off_v[r + 1];
+    const uint32_t b = off_v[r], e = off_v[r + 1];
     unsigned long long s = 0;
     for (uint32_t i = b + lane; i < e; i += 32) {
-      uint32_t u = adj_v[i];
+      const uint32_t u = adj_v[i];
       s += off_u[u + 1] - off_u[u];
     }
     for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(GMBE_FULL, s, o);
-    if (lane == 0) {
-      // issue key: wedges descending, then rank descending (ascending sort of the complements)
-      const uint32_t w = (uint32_t)(s > 0xffffffffull ? 0xffffffffull : s);
-      cost_key[r] = ((unsigned long long)(~w) << 32) | (~r);
-      atomicMax(&maxes[0], e - b);
-      atomicMax(&maxes[2], (uint32_t)(s > 0xffffffffull ? 0xffffffffull : s));
-      // root record: <= s candidates, each row of ceil(deg/32) words + id + k, padded to 4
-      const unsigned long long stride = (((e - b) + 31) / 32 + 2 + 3) & ~3ull;
-      atomicMax(rec_bound, s * stride);
-    }
+    // issue key: wedges descending, then rank descending (ascending sort of the complements)
+    const uint32_t w = (uint32_t)(s > 0xffffffffull ? 0xffffffffull : s);
+    if (lane == 0) cost_key[r] = ((unsigned long long)(~w) << 32) | (~r);
+    mdv = max(mdv, e - b);
+    mw = max(mw, w);
+    // root record: <= s candidates, each row of ceil(deg/32) words + id + k, padded to 4
+    const unsigned long long stride = (((e - b) + 31) / 32 + 2 + 3) & ~3ull;
+    mrec = max(mrec, s * stride);
   }
   for (uint32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < n_u; u += gridDim.x * blockDim.x)
-    atomicMax(&maxes[1], off_u[u + 1] - off_u[u]);
+    mdu = max(mdu, off_u[u + 1] - off_u[u]);
+  for (int o = 16; o; o >>= 1) {
+    mdv = max(mdv, __shfl_xor_sync(GMBE_FULL, mdv, o));
+    mdu = max(mdu, __shfl_xor_sync(GMBE_FULL, mdu, o));
+    mw = max(mw, __shfl_xor_sync(GMBE_FULL, mw, o));
+    mrec = max(mrec, (unsigned long long)__shfl_xor_sync(GMBE_FULL, mrec, o));
+  }
+  if (lane == 0) {
+    red[0][wib] = mdv;
+    red[1][wib] = mdu;
+    red[2][wib] = mw;
+    red[3][wib] = mrec;
+  }
+  __syncthreads();
+  if (threadIdx.x < 4) {
+    unsigned long long m = 0;
+    for (uint32_t k = 0; k < blockDim.x / 32; k++) m = max(m, red[threadIdx.x][k]);
+    if (threadIdx.x == 3) atomicMax(rec_bound, m);
+    else atomicMax(&maxes[threadIdx.x == 0 ? 0 : (threadIdx.x == 1 ? 1 : 2)], (uint32_t)m);
+  }
 }
 
 // stream-ordered allocations from the device's default pool (cheap to repeat per step)
@@ -160,6 +198,19 @@ cudaError_t radix_sort(Tmp& t, unsigned long long* in, unsigned long long* out, 
   e = t.alloc((char**)&tmp, bytes);
   if (e != cudaSuccess) return e;
   return cub::DeviceRadixSort::SortKeys(tmp, bytes, in, out, (int)n, 0, end_bit, s);
+}
+
+// stable LSD sort of (key, value) pairs on the low end_bit bits of the keys
+cudaError_t radix_sort_pairs(Tmp& t, const uint32_t* kin, uint32_t* kout, const uint32_t* vin, uint32_t* vout,
+                             uint64_t n, int end_bit, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  size_t bytes = 0;
+  cudaError_t e = cub::DeviceRadixSort::SortPairs(nullptr, bytes, kin, kout, vin, vout, (int)n, 0, end_bit, s);
+  if (e != cudaSuccess) return e;
+  void* tmp;
+  e = t.alloc((char**)&tmp, bytes);
+  if (e != cudaSuccess) return e;
+  return cub::DeviceRadixSort::SortPairs(tmp, bytes, kin, kout, vin, vout, (int)n, 0, end_bit, s);
 }
 
 cudaError_t excl_scan(Tmp& t, const uint32_t* in, uint32_t* out, uint64_t n, cudaStream_t s) {
@@ -241,7 +292,16 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   const uint32_t swapped = n_u < n_v ? 1u : 0u;
   const uint32_t NU = swapped ? n_v : n_u, NV = swapped ? n_u : n_v;
   const uint64_t m0 = n_edges;
-  // a1: ingest
+  const int bu = bits_for(NU), bv = bits_for(NV);  // NU / NV themselves fit (the sentinels below)
+  // Host-visible results of the build, read back by the call's ONE host synchronisation at the end:
+  // [0] bad id, [1] unique edges m, [2..4] Δ(V), Δ(U), wedge bound, [6..7] root-record bound (u64)
+  uint32_t* d_res;
+  TRY(t.alloc(&d_res, 8));
+  TRY(cudaMemsetAsync(d_res, 0, 8 * sizeof(uint32_t), s));
+  uint32_t* maxes = d_res + 2;
+  unsigned long long* d_recb = (unsigned long long*)(d_res + 6);
+  // a1: ingest -> (u << bv | v) keys -> sort -> dedupe flags (no host round trip: duplicates stay
+  // in place, flagged, and are squeezed out by the scatter below)
   const uint32_t* d_e = edges_uv;
   if (m0 && !o.edges_on_device) {
     uint32_t* tmp;
@@ -250,77 +310,56 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
     d_e = tmp;
   }
   unsigned long long *keys, *keys2;
-  int* d_bad;
   TRY(t.alloc(&keys, m0));
   TRY(t.alloc(&keys2, m0));
-  TRY(t.alloc(&d_bad, 1));
-  TRY(cudaMemsetAsync(d_bad, 0, sizeof(int), s));
-  if (m0) k_pack_edges<<<grid_for(m0), 256, 0, s>>>(d_e, m0, n_u, n_v, swapped, keys, d_bad), gmbe_note_launch();
+  if (m0) k_pack_edges<<<grid_for(m0), 256, 0, s>>>(d_e, m0, n_u, n_v, swapped, bv, keys, d_res), gmbe_note_launch();
   TRY(cudaGetLastError());
-  int h_bad = 0;
-  TRY(cudaMemcpyAsync(&h_bad, d_bad, sizeof(int), cudaMemcpyDeviceToHost, s));
-  TRY(cudaStreamSynchronize(s));
-  if (h_bad) return fail(gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: edge id out of range"));
-  TRY(radix_sort(t, keys, keys2, m0, 32 + bits_for(NU), s));
-  // unique
-  uint64_t m = 0;
-  if (m0) {
-    int* d_num;
-    TRY(t.alloc(&d_num, 1));
-    size_t bytes = 0;
-    TRY(cub::DeviceSelect::Unique(nullptr, bytes, keys2, keys, d_num, (int)m0, s));
-    char* tmp;
-    TRY(t.alloc(&tmp, bytes));
-    TRY(cub::DeviceSelect::Unique(tmp, bytes, keys2, keys, d_num, (int)m0, s));
-    int hn = 0;
-    TRY(cudaMemcpyAsync(&hn, d_num, sizeof(int), cudaMemcpyDeviceToHost, s));
-    TRY(cudaStreamSynchronize(s));
-    m = (uint64_t)hn;
-  }
-  // a2: degrees and order
-  uint32_t *deg_u, *deg_v, *deg_by_rank, *id2rank, *maxes;
+  TRY(radix_sort(t, keys, keys2, m0, bu + bv, s));
+  // a2: degrees of the unique edges and the global order
+  uint32_t *deg_u, *deg_v, *deg_by_rank, *id2rank, *flag, *pos;
   TRY(t.alloc(&deg_u, NU + 1));
   TRY(t.alloc(&deg_v, NV + 1));
   TRY(t.alloc(&deg_by_rank, NV + 1));
   TRY(t.alloc(&id2rank, NV + 1));
-  TRY(t.alloc(&maxes, 4));
-  unsigned long long* d_recb;
-  TRY(t.alloc(&d_recb, 1));
-  TRY(cudaMemsetAsync(d_recb, 0, 8, s));
+  TRY(t.alloc(&flag, m0));
+  TRY(t.alloc(&pos, m0));
   TRY(cudaMemsetAsync(deg_u, 0, (NU + 1) * sizeof(uint32_t), s));
   TRY(cudaMemsetAsync(deg_v, 0, (NV + 1) * sizeof(uint32_t), s));
   TRY(cudaMemsetAsync(deg_by_rank, 0, (NV + 1) * sizeof(uint32_t), s));
-  TRY(cudaMemsetAsync(maxes, 0, 4 * sizeof(uint32_t), s));
-  if (m) k_degrees<<<grid_for(m), 256, 0, s>>>(keys, m, deg_u, deg_v), gmbe_note_launch();
+  if (m0) k_unique_degrees<<<grid_for(m0), 256, 0, s>>>(keys2, m0, bv, flag, deg_u, deg_v), gmbe_note_launch();
+  if (m0) TRY(excl_scan(t, flag, pos, m0, s));
   unsigned long long *okeys, *okeys2;
   TRY(t.alloc(&okeys, NV));
   TRY(t.alloc(&okeys2, NV));
-  if (NV) k_order_keys<<<grid_for(NV), 256, 0, s>>>(deg_v, NV, o.order == GMBE_ORDER_IDENTITY, okeys), gmbe_note_launch();
-  TRY(radix_sort(t, okeys, okeys2, NV, 32 + bits_for(m + 1), s));
-  // persistent buffers
+  if (NV) k_order_keys<<<grid_for(NV), 256, 0, s>>>(deg_v, NV, o.order == GMBE_ORDER_IDENTITY, bv, okeys), gmbe_note_launch();
+  TRY(radix_sort(t, okeys, okeys2, NV, bv + bits_for(m0 + 1), s));
+  // persistent buffers (adjacency arrays sized m0 >= m; the tail past m holds the sentinels)
   uint32_t *off_v, *adj_v, *off_u, *adj_u, *rank2id;
   unsigned long long* hv;
   TRY(t.alloc(&off_v, NV + 1));
-  TRY(t.alloc(&adj_v, m));
+  TRY(t.alloc(&adj_v, m0));
   TRY(t.alloc(&off_u, NU + 1));
-  TRY(t.alloc(&adj_u, m));
+  TRY(t.alloc(&adj_u, m0));
   TRY(t.alloc(&rank2id, NV));
   TRY(t.alloc(&hv, NV));
   // library V side == caller V (hash side 1) unless swapped (then caller U, side 0)
   if (NV)
-    k_rank_maps<<<grid_for(NV), 256, 0, s>>>(okeys2, NV, swapped ? 0u : 1u, rank2id, id2rank, deg_v,
+    k_rank_maps<<<grid_for(NV), 256, 0, s>>>(okeys2, NV, bv, swapped ? 0u : 1u, rank2id, id2rank, deg_v,
                                              deg_by_rank, hv), gmbe_note_launch();
   TRY(excl_scan(t, deg_by_rank, off_v, (uint64_t)NV + 1, s));
   TRY(excl_scan(t, deg_u, off_u, (uint64_t)NU + 1, s));
-  if (m) {
-    unsigned long long *kv, *ku;
-    TRY(t.alloc(&kv, m));
-    TRY(t.alloc(&ku, m));
-    k_rekey<<<grid_for(m), 256, 0, s>>>(keys, m, id2rank, kv, ku), gmbe_note_launch();
-    TRY(radix_sort(t, kv, keys2, m, 32 + bits_for(NV), s));
-    k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_v), gmbe_note_launch();
-    TRY(radix_sort(t, ku, keys2, m, 32 + bits_for(NU), s));
-    k_low32<<<grid_for(m), 256, 0, s>>>(keys2, m, adj_u), gmbe_note_launch();
+  if (m0) {
+    // CSR_V (rank-major, u ascending) and CSR_U (u-major, ranks ascending) by two STABLE sorts on
+    // partial keys: the unique edges arrive u-major with v ascending; sorting them by rank alone
+    // keeps u ascending inside each rank; sorting that by u alone keeps ranks ascending inside each u
+    uint32_t *pk, *pv, *sk;
+    TRY(t.alloc(&pk, m0));
+    TRY(t.alloc(&pv, m0));
+    TRY(t.alloc(&sk, m0));
+    k_rank_pairs<<<grid_for(m0), 256, 0, s>>>(keys2, flag, pos, m0, bv, id2rank, NU, NV, pk, pv, d_res + 1),
+        gmbe_note_launch();
+    TRY(radix_sort_pairs(t, pk, sk, pv, adj_v, m0, bv, s));   // (rank, u): adj_v = the u's
+    TRY(radix_sort_pairs(t, adj_v, pv, sk, adj_u, m0, bu, s));  // (u, rank): adj_u = the ranks
   }
   uint32_t* issue;
   TRY(t.alloc(&issue, NV + 1));
@@ -333,11 +372,14 @@ extern "C" int gmbe_load_bipartite(uint32_t n_u, uint32_t n_v, const uint32_t* e
   TRY(radix_sort(t, ck, ck2, NV, 64, s));
   if (NV) k_issue<<<grid_for(NV), 256, 0, s>>>(ck2, NV, issue), gmbe_note_launch();
   TRY(cudaGetLastError());
-  uint32_t hm[4];
-  TRY(cudaMemcpyAsync(hm, maxes, sizeof(hm), cudaMemcpyDeviceToHost, s));
+  uint32_t hres[8];
+  TRY(cudaMemcpyAsync(hres, d_res, sizeof(hres), cudaMemcpyDeviceToHost, s));
+  TRY(cudaStreamSynchronize(s));  // the build's only host synchronisation
+  if (hres[0]) return fail(gmbe_set_error(GMBE_EINVAL, "gmbe_load_bipartite: edge id out of range"));
+  const uint64_t m = hres[1];
+  const uint32_t* hm = hres + 2;
   unsigned long long h_recb = 0;
-  TRY(cudaMemcpyAsync(&h_recb, d_recb, 8, cudaMemcpyDeviceToHost, s));
-  TRY(cudaStreamSynchronize(s));
+  std::memcpy(&h_recb, hres + 6, 8);
 
   void* keep[] = {off_v, adj_v, off_u, adj_u, rank2id, hv, issue};
   for (void* q : keep) {

@@ -816,3 +816,35 @@ def test_scheduler_variants_full_config(gmbe, name, sched):
         assert r.algo_bytes_cand == gd["algo_bytes_cand"]
     finally:
         g.free()
+
+
+# ---------------------------------------------------------------- chunked root claims
+def test_root_chunk_invariance(gmbe, dense_case):
+    """Warps claim root_chunk consecutive issue positions per atomic past the heavy head (local and
+    N1 shared cursor): any chunk size gives the same sets and canonical-tree counters."""
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        for ch in (1, 2, 7, 32, 1000):
+            r = g.enumerate(records=True, root_chunk=ch)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques), ch
+        cur = gmbe.SharedCursor.create(0)
+        try:
+            for k, ch in enumerate((1, 5, 32)):
+                a = g.enumerate(root_cursor=cur.slot_ptr(k), root_chunk=ch)
+                b = g.enumerate(root_cursor=cur.slot_ptr(k), root_chunk=ch)  # exhausted: nothing left
+                assert (a.count, a.checksum, b.count) == (o.count, o.checksum, 0)
+        finally:
+            cur.close()
+    finally:
+        g.free()
+    gd = _gold_cfg()["dblp"]
+    nu, nv, e = make_config("dblp")
+    g = gmbe.load(nu, nv, e)
+    try:
+        for ch in (1, 32):
+            r = g.enumerate(root_chunk=ch)
+            assert (r.count, r.checksum, r.nodes) == (gd["count"], int(gd["checksum"], 16), gd["nodes"])
+    finally:
+        g.free()
