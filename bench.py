@@ -86,24 +86,94 @@ def _traffic(name):
         return None
 
 
+def _profile(name):
+    """The committed full oracle run of a config (scripts/oracle_full.py): totals + per-root times."""
+    import numpy as np
+    pj = os.path.join(ROOT, "profiles", "oracle_full_%s.json" % name)
+    pz = os.path.join(ROOT, "profiles", "oracle_roots_%s.npz" % name)
+    try:
+        with open(pj) as f:
+            meta = json.load(f)
+        z = np.load(pz)
+        return meta, z["ns"].astype(np.float64) * 1e-9, z["count"]
+    except (OSError, KeyError, ValueError):
+        return None
+
+
+def _sample_mask(t, budget_s, lo=0.02, hi=2.0):
+    """A FIXED root sample of about budget_s seconds of oracle time (the same in every run and in both
+    bench arms): the roots whose profiled time lies in [lo, hi] s, every j-th of them in order of
+    internal id, j chosen so their profiled times add up to ~budget_s."""
+    import numpy as np
+    mid = np.nonzero((t >= lo) & (t <= hi))[0]
+    if len(mid) == 0:
+        return None
+    j = max(1, int(t[mid].sum() / budget_s))
+    m = np.zeros(len(t), bool)
+    m[mid[::j]] = True
+    return m
+
+
 def _cpu_sample(name, budget_s, gold):
-    """Time the oracle (as it stands, 1 thread) on a bounded sample of the workload: root shards
-    i/S (i = 0, 1, ...) of the degree-rank interleave, added until about budget_s of CPU time."""
+    """Time the oracle (as it stands, 1 thread) on a bounded, fixed root sample of the workload.
+
+    With a committed full oracle run of the config (profiles/oracle_full_<config>.json, per-root
+    times in oracle_roots_<config>.npz; scripts/oracle_full.py): the sample is fixed by that profile
+    (_sample_mask), and the whole job's per-core rate is estimated as the known count over the full
+    run's CPU time scaled by this host's speed on the sample (measured / profiled sample time).  The
+    oracle's per-root rates are far too heavy-tailed for a small sample's count/time to stand for the
+    job (on gh_work the top 100 of 55k roots hold 45% of its time).  Without a profile: root shards
+    i/S of the degree-rank interleave until about budget_s of CPU time (the raw sample rate).
+    Returns (value, detail dict)."""
+    import numpy as np
     import oracle
     from gmbe_inputs import make_config
     nu, nv, e = make_config(name)
+    prof = _profile(name)
+    if prof is not None:
+        meta, t, cnt = prof
+        mask = _sample_mask(t, budget_s)
+        if mask is not None:
+            t0 = time.time()
+            r = oracle.oracle_mbe(nu, nv, e, root_mask=mask, root_times=True)
+            wall = time.time() - t0
+            meas = float(r.per_root_ns[mask].sum()) * 1e-9
+            prof_s = float(t[mask].sum())
+            speed = meas / prof_s
+            full_s = float(t.sum()) * speed
+            value = meta["count"] / full_s
+            return value, {
+                "sample": "%d fixed roots (profiled 0.02-2 s each, %.1f s of the %.0f s full oracle run "
+                          "on %s) timed in %.1f s: host speed x%.3f of the profile -> whole job %.0f "
+                          "CPU-s; raw sample rate %.0f/s" % (
+                              int(mask.sum()), prof_s, float(t.sum()), meta.get("cpu_model", "?"), meas,
+                              1.0 / speed, full_s, r.count / max(meas, 1e-9)),
+                "method": "calibrated", "full_oracle_cpu_s_profile": meta.get("cpu_s"),
+                "profile_cores": meta.get("procs"), "sample_count": r.count, "sample_s": round(wall, 2)}
     if gold and gold.get("oracle_cpu_seconds"):
         shards = max(1, int(round(gold["oracle_cpu_seconds"] / budget_s)))
     else:
         shards = 1024
     count, dt, taken = 0, 0.0, 0
     while taken < shards and dt < budget_s:
-        t = time.time()
+        t0 = time.time()
         r = oracle.oracle_mbe(nu, nv, e, shard=(taken, shards))
-        dt += time.time() - t
+        dt += time.time() - t0
         count += r.count
         taken += 1
-    return count, dt, "root shards 0..%d of %d" % (taken - 1, shards)
+    return count / dt, {"sample": "root shards 0..%d of %d (%d bicliques, %.1f s)" % (taken - 1, shards, count, dt),
+                        "method": "raw"}
+
+
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 class ClockSampler:
@@ -145,30 +215,32 @@ class ClockSampler:
 
 
 def run_reference(a):
-    """Reference arm: the CPU oracle as it stands, on the host cores, same metric and workload."""
+    """Reference arm: the CPU oracle as it stands, on the host's cores, same metric and workload; each
+    step times the same fixed root sample as the main arm's cpu_baseline (_cpu_sample)."""
     ws, rank, _ = _dist()
     if rank != 0:
         return
     from gmbe_inputs import make_config
     gold = _gold(a.config)
     nu, nv, e = make_config(a.config)
+    per_step = min(a.cpu_budget_s, 180.0 / max(1, a.steps + min(a.warmup, 1)))  # whole run: a few minutes
     for _ in range(max(0, min(a.warmup, 1))):
-        _cpu_sample(a.config, 1.0, gold)
-    times, counts, sample = [], [], ""
-    per_step = min(a.cpu_budget_s, 180.0 / max(1, a.steps))  # whole run within a few minutes
+        _cpu_sample(a.config, per_step, gold)
+    vals, det = [], {}
     for _ in range(a.steps):
-        c, dt, sample = _cpu_sample(a.config, per_step, gold)
-        times.append(dt)
-        counts.append(c)
-    v = sum(counts) / sum(times)
+        v, det = _cpu_sample(a.config, per_step, gold)
+        vals.append(v)
+    v = statistics.median(vals)
     line = {"impl": "reference", "metric": _metric(a.config), "value": v, "unit": "bicliques/s",
             "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup,
-            "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
+            "ms_per_step": 1e3 * (gold["count"] / v if gold else 0.0), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": a.config, "n_u": nu, "n_v": nv, "m": int(len(e)),
-                       "sample": sample},
+                       "sample": det.get("sample")},
             "cpu_baseline": {"value": v, "unit": "bicliques/s", "cores": 1, "kind": "oracle",
-                             "sample": "oracle single-thread on %s of %s" % (sample, a.config)},
+                             "sample": "oracle single-thread, median of %d steps; %s" % (a.steps, det.get("sample")),
+                             "cpu_model": _cpu_model(), "host_cores": len(os.sched_getaffinity(0)),
+                             "step_values": [round(x, 1) for x in vals]},
             "e2e": {"value": v, "unit": "bicliques/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -370,10 +442,10 @@ def main():
             "clocks": clocks,
         }
         if ws == 1 and not a.no_cpu_baseline:
-            c, dt, sample = _cpu_sample(a.config, a.cpu_budget_s, gold)
-            line["cpu_baseline"] = {"value": c / dt, "unit": "bicliques/s", "cores": 1,
-                                    "kind": "oracle",
-                                    "sample": "%s (%d bicliques, %.1f s)" % (sample, c, dt)}
+            v, det = _cpu_sample(a.config, a.cpu_budget_s, gold)
+            line["cpu_baseline"] = {"value": v, "unit": "bicliques/s", "cores": 1, "kind": "oracle",
+                                    "sample": det["sample"], "method": det["method"],
+                                    "cpu_model": _cpu_model(), "host_cores": len(os.sched_getaffinity(0))}
         print(json.dumps(line), flush=True)
     if ws > 1:
         if dr is not None and rank != 0:

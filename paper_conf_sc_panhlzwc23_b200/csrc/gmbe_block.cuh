@@ -294,7 +294,8 @@ __global__ void __launch_bounds__(kBlkThreads, 1) k_enum_block(const Params P) {
   WarpMem M;
   M.keys = base;
   M.vals = (unsigned long long*)(base + P.tmax);
-  M.occ = base + 3ull * P.tmax;
+  M.bits = base + 3ull * P.tmax;
+  M.occ = M.bits + P.bmax;
   M.dyn = align4(M.occ + P.omax);
   M.dyn_end = base + P.arena_words;
   M.rbuf = P.rbuf ? P.rbuf + (uint64_t)gw * P.rbuf_words : nullptr;

@@ -68,7 +68,7 @@ struct Params {
   uint32_t* arena;    // per warp: keys[tmax] | vals[tmax] (u64) | occ[omax] | dynamic
   uint64_t arena_words;
   uint64_t col_budget;  // max words of a root's Γ-column store
-  uint32_t tmax, omax;
+  uint32_t tmax, omax, bmax;   // table slots, occupied-list words, rank-bitmap words
   uint32_t* rbuf;     // per-warp R-list stack (only with output)
   uint32_t rbuf_words;
   uint32_t* pool;     // task pool: subtasks and shared Γ columns, bump-allocated per call
@@ -90,7 +90,8 @@ struct Params {
                    // 16 = no thread-level tier (run_thr), 32 = path statistics into ctrl.phase,
                    // 64 = no suffix-mode roots, 128 = every root in suffix mode, 256 = no dense-mode roots,
                    // 512 = dense mode whenever the table can hold it, 1024 = build the roots only
-                   // (timing experiments: no subtree is walked, the result is incomplete)
+                   // (timing experiments: no subtree is walked, the result is incomplete),
+                   // 2048 = no register-resident tiny-root build (run_root_tiny)
   uint32_t donate;  // dynamic donation to idle warps (donate_reg)
   uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.thr_min)
   uint32_t split_wide;   // wide-universe split threshold on |C|·⌈|L|/32⌉ (opts.split_wide)
@@ -197,6 +198,7 @@ struct WarpMem {
   uint32_t* keys;               // clean hash table keys (EMPTY)
   unsigned long long* vals;     // clean hash table values (0)
   uint32_t* occ;                // occupied slots of the current root
+  uint32_t* bits;               // clean bitmap over the ranks (dense-mode roots' occupied ranks)
   uint32_t* skeys;              // the shared-memory table (kSmemTable slots)
   unsigned long long* svals;
   uint32_t* socc;
@@ -1710,6 +1712,7 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
           d = 0;
           dmask = 0;
         }
+        __syncwarp();  // the slots are read before any donor of a later step rewrites them
       }
     }
     if (!has) continue;
@@ -1844,14 +1847,17 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
       if (reg) {
         const bool st = split_mode && reg == top;  // heavy top: publish its children (run_reg)
 #ifndef GMBE_PROFILE
-        const unsigned long long n0 = A.get(kAcNodes);
+        const unsigned long long n0 = (P.debug & 32) ? A.get(kAcNodes) : 0ull;
 #endif
         const bool thr = !st && !(P.debug & 16) && run_thr(P, T, reg, lmap, A, ts, smem, reg_scratch, stack_hi);
         if (!thr) run_reg(P, T, reg, lmap, A, (RegLevel*)smem, reg_scratch, stack_hi, st, smem);
 #ifndef GMBE_PROFILE
-        if ((P.debug & 32) && lane == 0) {  // path statistics (experiments): jobs / nodes per tier
-          atomicAdd(&P.ctrl->phase[thr ? 0 : 2], 1ull);
-          atomicAdd(&P.ctrl->phase[thr ? 1 : 3], A.get(kAcNodes) - n0);
+        if (P.debug & 32) {  // path statistics (experiments): jobs / nodes per tier
+          const unsigned long long dn = A.get(kAcNodes) - n0;  // (a warp-wide shuffle)
+          if (lane == 0) {
+            atomicAdd(&P.ctrl->phase[thr ? 0 : 2], 1ull);
+            atomicAdd(&P.ctrl->phase[thr ? 1 : 3], dn);
+          }
         }
 #endif
         if (reg == top) return;
@@ -1962,6 +1968,119 @@ __device__ bool earlier_dominator(const DevGraph& g, const uint32_t* Lr, uint32_
 #define GMBE_SUFFIX_MIN 8192  // roots with at least this many wedges may scan only later ranks
 #endif
 
+// Tiny roots (|L_r| <= 32 and <= 32 wedges: most roots of light-tailed graphs such as the DBLP
+// shape) are built entirely in registers: lane p holds wedge p = (u_i, v) after one scan of the
+// degrees; __match_any_sync groups the wedges by v, so a group leader knows k(v) = |N(v) ∩ L_r| (its
+// group size) and the row N(v) ∩ L_r (an OR-reduction over the group) without a hash table, an
+// occupied list, a sort or a table clean-up.  Classification (Alg 3 L3-7), emission, the Γ index
+// (X2 rows) and the candidate record (rank order by counting smaller candidates) are then the same
+// as run_root's, written straight to the warp's dynamic region.  lane j < l: (beg, deg) of N(u_j).
+__device__ bool run_root_tiny(const Params& P, uint32_t r, uint32_t l, const uint32_t* Lr, uint32_t beg,
+                              uint32_t deg, uint32_t wedges, WarpMem& M, Acc& A, TaskCtx& Tc, uint32_t** top,
+                              uint32_t** lo) {
+  const uint32_t lane = lane_id();
+  const DevGraph& g = P.g;
+  // wedge p -> (i, v): owner i by a binary search over the exclusive degree prefix
+  uint32_t inc = deg;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t t = __shfl_up_sync(GMBE_FULL, inc, o);
+    if (lane >= (uint32_t)o) inc += t;
+  }
+  const uint32_t excl = inc - deg;
+  uint32_t own = 0;
+#pragma unroll
+  for (int st = 16; st; st >>= 1) {
+    const uint32_t cand = own + st;
+    const uint32_t e = __shfl_sync(GMBE_FULL, excl, cand & 31);
+    if (cand < l && e <= lane) own = cand;
+  }
+  const uint32_t ob = __shfl_sync(GMBE_FULL, beg, own), oe = __shfl_sync(GMBE_FULL, excl, own);
+  const bool act0 = lane < wedges;
+  const uint32_t v = act0 ? __ldg(g.adj_u + ob + lane - oe) : kNone;
+  const bool act = act0 && v != r;
+  const uint32_t peers = __match_any_sync(GMBE_FULL, act ? v : kNone - 1 - lane);
+  const uint32_t k = __popc(peers);
+  const uint32_t row = __reduce_or_sync(peers, 1u << own);  // N(v) ∩ L_r over the universe
+  const bool leader = act && lane == (uint32_t)(__ffs(peers) - 1);
+  // Alg 3 L3-7: k == |L| -> R (skip the root unless v_s is R's earliest vertex); later -> C
+  const bool isR = leader && k == l;
+  if (__any_sync(GMBE_FULL, isR && v < r)) return false;
+  const bool isC = leader && k < l && v > r;
+  const bool isX = leader && k >= 2;  // X2: can cover an L' with |L'| >= 2
+  const unsigned long long hv_r = g.hv[r];
+  const unsigned long long hvx = isR ? g.hv[v] : 0ull;
+  const unsigned long long sl = warp_sum64r(lane < l ? hash_u(P, Lr[lane]) : 0ull);
+  const unsigned long long sr = warp_sum64r(hvx) + hv_r;
+  const uint32_t bR = __ballot_sync(GMBE_FULL, isR), bC = __ballot_sync(GMBE_FULL, isC),
+                 bX = __ballot_sync(GMBE_FULL, isX);
+  const uint32_t nR = __popc(bR), nC = __popc(bC), nx = __popc(bX);
+  uint32_t* gx = align4(M.dyn);
+  uint32_t* rec = align4(gx + 4 + 2 * nx + r4(nx));
+  if (!fits(P, rec + kHdr + 4 + 4 * nC + 64, M.dyn_end)) return false;
+  A.add(kAcRootsRun, 1);
+  A.add(kAcCount, 1);  // emit (L_r, R_r) (A5)
+  A.add(kAcChecksum, pair_hash(P, sl, sr));
+  if (P.per_root && lane == 0) atomicAdd(P.per_root + r, 1ull);
+  if (M.rbuf) {
+    if (lane == 0) M.rbuf[0] = r;
+    if (isR) M.rbuf[1 + __popc(bR & lanemask_lt())] = v;
+    __syncwarp();
+    if (P.out_ids || P.sring) write_record(P, nullptr, 0, nullptr, Lr, l, M.rbuf, nR + 1);
+  }
+  if (nC == 0) return false;
+  // Γ index (universe <= 32 bits, |X2| <= 32: the rows are lane-resident in every task of the root)
+  if (lane == 0) {
+    gx[0] = nx;
+    gx[1] = l;
+  }
+  if (isX) {
+    const uint32_t xp = __popc(bX & lanemask_lt());
+    ((unsigned long long*)(gx + 4))[xp] = row;
+    gx[4 + 2 * nx + xp] = v;
+  }
+  // the root's node record: candidates in rank order (a candidate's position = smaller candidates)
+  uint32_t pos = 0;
+  for (uint32_t m = bC; m; m &= m - 1) pos += __shfl_sync(GMBE_FULL, v, __ffs(m) - 1) < v;
+  if (isC) ((uint4*)(rec + kHdr + 4))[pos] = make_uint4(row, v, k, 0);
+  if (lane < 4) rec[kHdr + lane] = lane == 0 ? (l >= 32 ? GMBE_FULL : (1u << l) - 1u) : 0u;
+  if (lane == 0) {
+    rec[0] = nC;
+    rec[1] = 0;
+    rec[2] = l;
+    rec[3] = 0;
+    rec[4] = kNone;
+    rec[5] = nR + 1;
+    rec[6] = (uint32_t)sr;
+    rec[7] = (uint32_t)(sr >> 32);
+  }
+  __syncwarp();
+  Tc.map = Lr;
+  Tc.W = 1;
+  Tc.W4 = 4;
+  Tc.E = 4;
+  Tc.root = r;
+  Tc.rlist = M.rbuf;
+  Tc.cols = nullptr;
+  Tc.gx = gx;
+  Tc.ncw = 0;
+  Tc.auxref = 0;
+  if (heavy(P, l, nC)) {  // the root will be split: share its Γ index with the subtasks
+    const uint32_t words = 4 + 2 * nx + r4(nx);
+    const uint32_t co = pool_alloc(P, r4(words));
+    if (co != kNone) {
+      uint32_t* cp = pool_ptr(P, co);
+      for (uint32_t j = lane; j < words; j += 32) cp[j] = gx[j];
+      __syncwarp();
+      Tc.gx = cp;
+      Tc.auxref = co + 1;
+    }
+  }
+  *top = rec;
+  *lo = align4(rec + kHdr + 4 + 4 * nC);
+  return true;
+}
+
 // Root v_s (rank r): L_r = N(v_s); wedge scan of N2(v_s) with k(v) = |N(v) ∩ L_r|.  Emits the root
 // biclique and, if it has candidates, prepares its node record as a task (Tc, *top, stack from *lo)
 // for the caller's single dispatch site; returns whether it did.
@@ -1972,13 +2091,17 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   if (l == 0) return false;  // isolated vertex: in no biclique (A17)
   const uint32_t* Lr = g.adj_v + lb;
   const unsigned long long hv_r = g.hv[r];  // issued early, consumed at the root's emission
-  uint32_t wp = 0;
+  uint32_t wp = 0, beg0 = 0;  // (lane j < 32: beg0 / wp = N(u_j) of the first 32 members)
   for (uint32_t j = lane; j < l; j += 32) {
     const uint32_t u = Lr[j];
-    wp += g.off_u[u + 1] - g.off_u[u];
+    const uint32_t b = g.off_u[u], d = g.off_u[u + 1] - b;
+    if (j < 32) beg0 = b;
+    wp += d;
   }
   const uint32_t wedges = warp_sum(wp);
   A.add(kAcAbytes, 4ull * (l + wedges));
+  if (l <= 32 && wedges <= 32 && !(P.debug & (128 | 2048)))  // tiny root: register-resident build
+    return run_root_tiny(P, r, l, Lr, beg0, wp, wedges, M, A, Tc, top, lo);
   // Suffix mode (B200 addition, reading B5): a root with many wedges but few of them to
   // later-ranked vertices (high degree rank: few candidates, huge excluded set) counts k only over
   // the rank suffix of each list; the skip test (Alg 3 L7) then looks for an earlier dominator
@@ -2024,36 +2147,46 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   // slots).  Pass 1 is then fire-and-forget atomics (no probing), and the occupied list comes from
   // a scan of the rank range -- in rank order, so the candidates need no sort.
   const uint32_t lo_v = after != kNone ? r + 1 : 0u;
+  // The occupied ranks are marked in a per-warp bitmap as well (fire-and-forget atomics), so the
+  // scan for them reads (n_v - lo_v)/32 words instead of the whole value range.
   const bool dense = !stab && g.n_v <= P.tmax && !(P.debug & 256) &&
                      ((uint64_t)(g.n_v - lo_v) <= (uint64_t)GMBE_DENSE_RATIO * scanned || (P.debug & 512));
   PH_START(A);
   // pass 1 (Alg 3 L2-3)
   uint32_t nocc = 0;
   if (dense) {
+    uint32_t* bits = M.bits;
     for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
       if (act && v != r) {
         if (small) atomicOr(vals + v, 1ull << i);
         else atomicAdd(vals + v, 1ull);
+        atomicOr(bits + (v >> 5), 1u << (v & 31));
       }
     }, after);
     __syncwarp();
     __threadfence();
-    for (uint32_t b = lo_v; b < g.n_v; b += 256) {
-      unsigned long long x[8];
+    // occupied ranks from the bitmap, in rank order; the words are cleared behind the scan
+    const uint32_t wend = (g.n_v + 31) >> 5;
+    for (uint32_t wb = lo_v >> 5; wb < wend; wb += 64) {
+      const uint32_t w0 = wb + lane, w1 = wb + 32 + lane;
+      const uint32_t x0 = w0 < wend ? __ldcg(bits + w0) : 0u;  // L2: pass 1 wrote with atomics
+      const uint32_t x1 = w1 < wend ? __ldcg(bits + w1) : 0u;
+      if (x0) bits[w0] = 0u;
+      if (x1) bits[w1] = 0u;
 #pragma unroll
-      for (int q = 0; q < 8; q++) {
-        const uint32_t v = b + q * 32 + lane;
-#if GMBE_DENSE_CS
-        x[q] = v < g.n_v ? __ldcs(vals + v) : 0ull;  // streaming (evict-first): a one-pass scan
-#else
-        x[q] = v < g.n_v ? __ldcg(vals + v) : 0ull;  // L2: pass 1 wrote with atomics
-#endif
-      }
+      for (int h = 0; h < 2; h++) {
+        uint32_t x = h ? x1 : x0;
+        const uint32_t c = __popc(x);
+        uint32_t incl = c;
 #pragma unroll
-      for (int q = 0; q < 8; q++) {
-        const uint32_t bal = __ballot_sync(GMBE_FULL, x[q] != 0ull);
-        if (x[q]) occl[nocc + __popc(bal & lanemask_lt())] = b + q * 32 + lane;
-        nocc += __popc(bal);
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t t = __shfl_up_sync(GMBE_FULL, incl, o);
+          if (lane >= (uint32_t)o) incl += t;
+        }
+        uint32_t q = nocc + incl - c;
+        const uint32_t base = (h ? w1 : w0) << 5;
+        for (; x; x &= x - 1) occl[q++] = base + __ffs(x) - 1;
+        nocc += __shfl_sync(GMBE_FULL, incl, 31);
       }
     }
     __syncwarp();
@@ -2371,7 +2504,8 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
   WarpMem M;
   M.keys = base;
   M.vals = (unsigned long long*)(base + P.tmax);
-  M.occ = base + 3ull * P.tmax;
+  M.bits = base + 3ull * P.tmax;
+  M.occ = M.bits + P.bmax;
   M.dyn = align4(M.occ + P.omax);
   M.dyn_end = base + P.arena_words;
   M.rbuf = P.rbuf ? P.rbuf + (uint64_t)gw * P.rbuf_words : nullptr;
@@ -2396,10 +2530,9 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
     uint32_t* lo = M.dyn;
     uint32_t lmap = 0, kind = 2, item = 0, tl_l = 0, tl_c = 0;
     const long long c0 = P.per_root_cycles ? clock64() : 0;
-    const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = A.get(kAcNodes);
+    const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = P.timeline ? A.get(kAcNodes) : 0ull;
     uint32_t task = kNone;
-    // the queue is polled between root chunks (inside a chunk of light roots the warp keeps going)
-    if (lane == 0 && ck_pos == ck_end) task = queue_pop(P);
+    if (lane == 0) task = queue_pop(P);  // split subtasks first (Alg 4 L3), also inside a root chunk
     task = __shfl_sync(GMBE_FULL, task, 0);
     bool release = true;  // this item ends a unit of `pending` (a task, or a chunk's last root)
     if (task != kNone) {
@@ -2512,9 +2645,9 @@ struct Workspace {
   int device = -1;
   void* arena = nullptr;
   size_t arena_bytes = 0;
-  uint64_t layout[4] = {0, 0, 0, 0};  // tmax, omax, arena_words, nwarps of the clean tables
+  uint64_t layout[5] = {0, 0, 0, 0, 0};  // tmax, omax, arena_words, nwarps, bmax of the clean tables
   bool clean = false;
-  uint64_t tmax = 0, omax = 0, dyn = 0, nwarps = 0, pool_auto = 0;  // cached sizing
+  uint64_t tmax = 0, omax = 0, bmax = 0, dyn = 0, nwarps = 0, pool_auto = 0;  // cached sizing
   bool dyn_capped = false;
   int sms = 0, bps_max = 0, bps_max_blk = 0;
   void* pool = nullptr;
@@ -2681,29 +2814,32 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   const uint64_t wb = (uint64_t)g.wedge_bound + 64;
   uint64_t tmax = 64;
   while (tmax < 2 * wb) tmax <<= 1;
+  const uint64_t bmax = ((uint64_t)(g.n_v + 31) / 32 + 3) & ~3ull;  // rank bitmap of dense-mode roots
   uint64_t omax = (wb + 3) & ~3ull;
   const uint64_t cols_bound = std::min<uint64_t>((uint64_t)g.delta_v * (wb / 32 + 1), 1u << 21);
   const uint64_t dyn_want = o.arena_words ? o.arena_words
                                           : (uint64_t)g.rec_bound * 4 + 4 * wb + 2 * cols_bound + (1u << 18);
   uint64_t arena_words;
-  bool reuse = W.arena && W.nwarps == nwarps && W.tmax >= tmax && W.omax >= omax &&
+  bool reuse = W.arena && W.nwarps == nwarps && W.tmax >= tmax && W.omax >= omax && W.bmax >= bmax &&
                (W.dyn >= dyn_want || (!o.arena_words && W.dyn_capped));
   if (reuse && W.dyn < dyn_want) {
     // a layout capped by free memory at an earlier call: re-size if there is more room now
     size_t fr = 0, tot = 0;
     GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
     fr += W.arena_bytes;
-    const uint64_t fixed = 3 * W.tmax + W.omax + 8;
+    const uint64_t fixed = 3 * W.tmax + W.bmax + W.omax + 8;
     const uint64_t cap_total = (uint64_t)(fr * 0.5) / 4 / nwarps;
     const uint64_t cap_now = cap_total > fixed ? cap_total - fixed : 0;
     if (cap_now > W.dyn + W.dyn / 8) reuse = false;
   }
+  uint64_t bmax_use = bmax;
   if (reuse) {
     tmax = W.tmax;
     omax = W.omax;
+    bmax_use = W.bmax;
     arena_words = W.layout[2];
   } else {
-    const uint64_t fixed = 3 * tmax + omax + 8;
+    const uint64_t fixed = 3 * tmax + bmax + omax + 8;
     uint64_t dyn = dyn_want;
     bool capped = false;
     if (!o.arena_words) {
@@ -2720,6 +2856,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
     arena_words = (fixed + dyn + 3) & ~3ull;
     W.tmax = tmax;
     W.omax = omax;
+    W.bmax = bmax;
     W.dyn = dyn;
     W.dyn_capped = capped;
     W.nwarps = nwarps;
@@ -2749,17 +2886,18 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
       (void)cudaGetLastError();
       W.dyn = std::max<uint64_t>(W.dyn / 2, 1u << 16);
       W.dyn_capped = true;
-      arena_words = (3 * tmax + omax + 8 + W.dyn + 3) & ~3ull;
+      arena_words = (3 * tmax + bmax_use + omax + 8 + W.dyn + 3) & ~3ull;
       ae = ensure(&W.arena, &W.arena_bytes, nwarps * arena_words * 4);
     }
     GMBE_CUDA_TRY(ae);
   }
   {
-    const uint64_t sig[4] = {tmax, omax, arena_words, nwarps};
+    const uint64_t sig[5] = {tmax, omax, arena_words, nwarps, bmax_use};
     if (!W.clean || std::memcmp(sig, W.layout, sizeof(sig)) != 0) {
       // keys := EMPTY, vals := 0 -- once; every root leaves its slots clean again
       GMBE_CUDA_TRY(cudaMemset2DAsync(W.arena, arena_words * 4, 0xff, tmax * 4, nwarps, s));
-      GMBE_CUDA_TRY(cudaMemset2DAsync((uint32_t*)W.arena + tmax, arena_words * 4, 0, 2 * tmax * 4, nwarps, s));
+      GMBE_CUDA_TRY(cudaMemset2DAsync((uint32_t*)W.arena + tmax, arena_words * 4, 0, (2 * tmax + bmax_use) * 4,
+                                      nwarps, s));
       std::memcpy(W.layout, sig, sizeof(sig));
       W.clean = true;
     }
@@ -2806,6 +2944,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   P.col_budget = W.dyn / 2;
   P.tmax = (uint32_t)tmax;
   P.omax = (uint32_t)omax;
+  P.bmax = (uint32_t)bmax_use;
   P.rbuf = want_out ? (uint32_t*)W.rbuf : nullptr;
   P.rbuf_words = rbuf_words;
   P.pool = (uint32_t*)W.pool;
