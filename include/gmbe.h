@@ -161,9 +161,10 @@ typedef struct {
    *     roots, so counts / checksums add (mod 2^64). */
   uint32_t part_mode;
   uint32_t root_chunk;    /* root positions a warp claims per atomic once past the first 1/8 (the
-                             heavy head) of the issue list: 0 = default 16, 1 = one root per atomic,
-                             at most 32.  Fewer atomics on the (local or N1 shared) root cursor; the
-                             result and the canonical-tree counters do not depend on it. */
+                             heavy head) of the issue list: 0 = default 1 (one root per atomic),
+                             at most 32.  Fewer atomics on the (local or N1 shared) root cursor --
+                             e.g. 16 for light-root graphs under N1; the result and the
+                             canonical-tree counters do not depend on it. */
 } gmbe_opts;
 
 enum { GMBE_PART_INTERLEAVE = 0, GMBE_PART_COST = 1 };

@@ -1488,7 +1488,7 @@ __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const
 #define GMBE_THR_DONATE_MASK 3  // run_thr checks ctrl.hungry every (mask + 1) steps
 #endif
 #ifndef GMBE_ROOT_CHUNK
-#define GMBE_ROOT_CHUNK 16  // light roots claimed per atomic (opts.root_chunk)
+#define GMBE_ROOT_CHUNK 1  // light roots claimed per atomic (opts.root_chunk); >1 measured slower on the heavy-tailed shapes
 #endif
 #ifndef GMBE_THR_MIN_EST
 #define GMBE_THR_MIN_EST 16  // jobs with fewer adjacency bits (Σ(k-1)) stay on run_reg (setup > work)
@@ -1546,10 +1546,9 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
   const unsigned long long* xrow = (const unsigned long long*)(T.gx + 4);
   const uint32_t* xid = T.gx + 4 + 2 * nx;
   bool over = false;
-  for (uint32_t b = 0; b < nx; b += 32) {
-    const uint32_t x = b + lane;
-    const unsigned long long p = x < nx ? xrow[x] & L0 : 0ull;
-    bool q = __popcll(p) >= 2 && p != L0;
+  auto consider = [&](uint32_t x, bool in, uint32_t first) {
+    const unsigned long long p = in ? xrow[x] & L0 : 0ull;
+    bool q = __popcll(p) >= 2 && p != L0 && (first >= 64 || (uint32_t)(__ffsll(p) - 1) == first);
     if (q) q = !sorted_has(ts->id, nC, xid[x]);
     if (q) {  // insert p (linear probing; 0 = empty)
       uint32_t h = (uint32_t)((p * 0x9E3779B97F4A7C15ull) >> 57), n = 0;
@@ -1563,6 +1562,24 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
         }
       }
     }
+  };
+  // X2 vertices touching >= 2 members of L0: scan all of X2, or -- when the per-vertex X2 lists of
+  // the members of L0 are shorter in total -- walk those lists (x taken from the list of its first
+  // member in L0 only)
+  const uint32_t listed = nx > 64 ? warp_sum(((L0 >> lane) & 1ull ? T.gl0 : 0u) + ((L0 >> (lane + 32)) & 1ull ? T.gl1 : 0u))
+                                  : kNone;
+  if (listed < nx) {
+    for (unsigned long long m = L0; m; m &= m - 1) {
+      const uint32_t j = __ffsll(m) - 1;
+      const uint32_t off = __shfl_sync(GMBE_FULL, j < 32 ? T.go0 : T.go1, j & 31);
+      const uint32_t len = __shfl_sync(GMBE_FULL, j < 32 ? T.gl0 : T.gl1, j & 31);
+      for (uint32_t b = 0; b < len; b += 32) {
+        const bool in = b + lane < len;
+        consider(in ? T.gxl[off + b + lane] : 0u, in, j);
+      }
+    }
+  } else {
+    for (uint32_t b = 0; b < nx; b += 32) consider(b + lane, b + lane < nx, 64);
   }
   __syncwarp();
   if (__any_sync(GMBE_FULL, over)) return false;
@@ -2987,7 +3004,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   if (o.scheduler == GMBE_SCHED_WARP) P.debug |= 16;  // one warp per node: no thread-level tier
   P.thr_min_est = o.thr_min ? o.thr_min : GMBE_THR_MIN_EST;
   // root claims: after the heavy head of the issue list (the first 1/8 of the positions, one root
-  // per atomic), a warp claims root_chunk consecutive positions per atomic (default 16, <= 32)
+  // per atomic), a warp claims root_chunk consecutive positions per atomic (default 1, <= 32)
   P.chunk = o.root_chunk ? std::min<uint32_t>(o.root_chunk, 32u) : GMBE_ROOT_CHUNK;
   P.chunk_from = P.n_roots / 8;
   P.split_wide = o.split_wide ? o.split_wide : GMBE_SPLIT_WIDE;
