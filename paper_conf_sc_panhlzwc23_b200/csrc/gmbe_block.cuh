@@ -308,7 +308,12 @@ __global__ void __launch_bounds__(kBlkThreads, 1) k_enum_block(const Params P) {
     M.svals[j] = 0;
   }
   __syncthreads();
-  Acc A = {};
+  Acc A;  // the block's counters: held (and updated) by warp 0, one per lane, flushed at exit
+  A.v = 0;
+#ifdef GMBE_PROFILE
+  for (int k = 0; k < 16; k++) A.ph[k] = 0;
+  A.t0 = 0;
+#endif
   while (true) {
     if (tid == 0) {
       const unsigned long long t =

@@ -113,6 +113,7 @@ struct Acc {
     asm("mov.u32 %0, %%laneid;" : "=r"(l));
     if (l == k) v += x;
   }
+  // counter k (a warp-wide shuffle: every lane must call it)
   __device__ __forceinline__ unsigned long long get(uint32_t k) const {
     const uint32_t lo = __shfl_sync(0xffffffffu, (uint32_t)v, k), hi = __shfl_sync(0xffffffffu, (uint32_t)(v >> 32), k);
     return ((unsigned long long)hi << 32) | lo;
@@ -1487,6 +1488,9 @@ __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const
 #ifndef GMBE_THR_DONATE_MASK
 #define GMBE_THR_DONATE_MASK 3  // run_thr checks ctrl.hungry every (mask + 1) steps
 #endif
+#ifndef GMBE_TINY_REDUX
+#define GMBE_TINY_REDUX 0  // tiny roots: rows by per-group OR-reduction (1) or one ballot per member (0)
+#endif
 #ifndef GMBE_ROOT_CHUNK
 #define GMBE_ROOT_CHUNK 1  // light roots claimed per atomic (opts.root_chunk); >1 measured slower on the heavy-tailed shapes
 #endif
@@ -1631,6 +1635,10 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
   ThrLevel stk[32];
   bool has = lane == 0;
   unsigned long long L = L0, SR = ((unsigned long long)rec[7] << 32) | rec[6];
+  // SL = Σ_{u∈L} hU(u) of the lane's current node, kept incrementally (children subtract the members
+  // they drop, pops add them back), so the maximality loop can stop as soon as L' is proven maximal
+  unsigned long long SL = 0;
+  for (unsigned long long m = L0; m; m &= m - 1) SL += cols[__ffsll(m) - 1].hu;
   const uint32_t cand_all = nC >= 32 ? GMBE_FULL : ((1u << nC) - 1u);
   uint32_t C = cand_all, next = 0, Rm = 0, d = 0, dmask = 0;
   uint32_t bd = 0;  // tree depth (below the job's top) of this lane's level 0
@@ -1654,7 +1662,9 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
         const uint32_t rmp = stk[d].Rm, diff = Rm & ~rmp;  // {i} ∪ absorbed of the finished child
         next = __ffs(diff);
         for (uint32_t m = diff; m; m &= m - 1) SR -= ts->hv[__ffs(m) - 1];
-        L = stk[d].L;
+        const unsigned long long lpar = stk[d].L;
+        for (unsigned long long m = lpar & ~L; m; m &= m - 1) SL += cols[__ffsll(m) - 1].hu;
+        L = lpar;
         C = stk[d].C;
         Rm = rmp;
         dmask &= ~(1u << d);
@@ -1728,6 +1738,8 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
           bd = (uint32_t)(o[3] >> 32);
           d = 0;
           dmask = 0;
+          SL = 0;
+          for (unsigned long long m = L; m; m &= m - 1) SL += cols[__ffsll(m) - 1].hu;
         }
         __syncwarp();  // the slots are read before any donor of a later step rewrites them
       }
@@ -1775,22 +1787,20 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
       sl = cols[j].hu;
     } else {  // |L'| >= 2: no Q pattern and no job candidate outside R' may cover L'
       const uint32_t outside = cand_all & ~(Rm | (1u << i) | ab);
-      unsigned long long qa = ~0ull, m = lp;
+      unsigned long long qa = ~0ull;
       uint32_t ca = GMBE_FULL;
-      for (; m; m &= m - 1) {
+      for (unsigned long long m = lp; m; m &= m - 1) {
         const uint32_t j = __ffsll(m) - 1;
-        const ThrCol tc = cols[j];
-        qa &= tc.q;
-        sl += tc.hu;
+        qa &= cols[j].q;
         ca &= ts->ccol[j];
-        if (!qa && !(ca & outside)) {
-          m &= m - 1;
-          break;
-        }
+        if (!qa && !(ca & outside)) break;
       }
       maximal = !qa && !(ca & outside);
-      if (maximal)
-        for (; m; m &= m - 1) sl += cols[__ffsll(m) - 1].hu;
+      // SL(L') from the node's SL(L): remove the members L' dropped (usually a few)
+      if (maximal) {
+        sl = SL;
+        for (unsigned long long m = L & ~lp; m; m &= m - 1) sl -= cols[__ffsll(m) - 1].hu;
+      }
     }
     if (!maximal) {
       n_nonmax++;
@@ -1815,6 +1825,7 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     d++;
     L = lp;
     SR = srn;
+    SL = sl;
     C = cd;
     Rm = rmn;
     next = 0;
@@ -2018,7 +2029,15 @@ __device__ bool run_root_tiny(const Params& P, uint32_t r, uint32_t l, const uin
   const bool act = act0 && v != r;
   const uint32_t peers = __match_any_sync(GMBE_FULL, act ? v : kNone - 1 - lane);
   const uint32_t k = __popc(peers);
-  const uint32_t row = __reduce_or_sync(peers, 1u << own);  // N(v) ∩ L_r over the universe
+  // the row N(v) ∩ L_r over the universe: bit i iff a wedge of u_i is in v's group (one ballot per
+  // member -- a per-group OR-reduction would serialise over the groups)
+#if GMBE_TINY_REDUX
+  const uint32_t row = __reduce_or_sync(peers, 1u << own);
+#else
+  uint32_t row = 0;
+  for (uint32_t i = 0; i < l; i++)
+    if (peers & __ballot_sync(GMBE_FULL, act0 && own == i)) row |= 1u << i;
+#endif
   const bool leader = act && lane == (uint32_t)(__ffs(peers) - 1);
   // Alg 3 L3-7: k == |L| -> R (skip the root unless v_s is R's earliest vertex); later -> C
   const bool isR = leader && k == l;
@@ -2509,16 +2528,13 @@ __device__ __forceinline__ unsigned long long tl_info(unsigned long long nodes, 
 #define GMBE_WPB 8  // warps per block
 #endif
 constexpr uint32_t kWpb = GMBE_WPB;
-__global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const Params P) {
-  __shared__ unsigned long long s_sort[kWpb][kSmemSort];
-  __shared__ unsigned long long s_tvals[kWpb][kSmemTable ? kSmemTable : 1];
-  __shared__ uint32_t s_tkeys[kWpb][kSmemTable ? kSmemTable : 1];
-  __shared__ uint32_t s_tocc[kWpb][kSmemTable ? kSmemTable / 2 : 1];
-  __shared__ ThrSmem s_thr[kWpb];
-  const uint32_t lane = lane_id();
-  const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  uint32_t* base = P.arena + (uint64_t)gw * P.arena_words;
+// The warp's memory: its arena slice (clean hash table, rank bitmap, occupied list, dynamic region)
+// and its shared-memory slices -- recomputed where needed instead of held across the persistent loop
+// (long-lived pointers were the loop's main register spills).
+__device__ __forceinline__ WarpMem warp_mem(const Params& P, uint32_t gw, unsigned long long* sm_sort,
+                                           uint32_t* skeys, unsigned long long* svals, uint32_t* socc) {
   WarpMem M;
+  uint32_t* base = P.arena + (uint64_t)gw * P.arena_words;
   M.keys = base;
   M.vals = (unsigned long long*)(base + P.tmax);
   M.bits = base + 3ull * P.tmax;
@@ -2526,31 +2542,64 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
   M.dyn = align4(M.occ + P.omax);
   M.dyn_end = base + P.arena_words;
   M.rbuf = P.rbuf ? P.rbuf + (uint64_t)gw * P.rbuf_words : nullptr;
-  M.sm_sort = s_sort[threadIdx.x >> 5];
-  M.skeys = s_tkeys[threadIdx.x >> 5];
-  M.svals = s_tvals[threadIdx.x >> 5];
-  M.socc = s_tocc[threadIdx.x >> 5];
+  M.sm_sort = sm_sort;
+  M.skeys = skeys;
+  M.svals = svals;
+  M.socc = socc;
+  return M;
+}
+
+__global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const Params P) {
+  __shared__ unsigned long long s_sort[kWpb][kSmemSort];
+  __shared__ unsigned long long s_tvals[kWpb][kSmemTable ? kSmemTable : 1];
+  __shared__ uint32_t s_tkeys[kWpb][kSmemTable ? kSmemTable : 1];
+  __shared__ uint32_t s_tocc[kWpb][kSmemTable ? kSmemTable / 2 : 1];
+  __shared__ ThrSmem s_thr[kWpb];
+  const uint32_t lane = lane_id();
+#define GMBE_WARP_MEM()                                                                                      \
+  warp_mem(P, (blockIdx.x * blockDim.x + threadIdx.x) >> 5, s_sort[threadIdx.x >> 5], s_tkeys[threadIdx.x >> 5], \
+           s_tvals[threadIdx.x >> 5], s_tocc[threadIdx.x >> 5])
   for (uint32_t j = lane; j < kSmemTable; j += 32) {
-    M.skeys[j] = GMBE_EMPTY;
-    M.svals[j] = 0;
+    s_tkeys[threadIdx.x >> 5][j] = GMBE_EMPTY;
+    s_tvals[threadIdx.x >> 5][j] = 0;
   }
   __syncwarp();
-  Acc A = {};
+  Acc A;
+  A.v = 0;
+#ifdef GMBE_PROFILE
+  for (int k = 0; k < 16; k++) A.ph[k] = 0;
+  A.t0 = 0;
+#endif
   bool roots_done = false, is_hungry = false;
   uint32_t idle = 0;
-  uint32_t ck_pos = 0, ck_end = 0, ck_base = 0, ck_rk = 0, ck_lb = 0, ck_l = 0;  // claimed root chunk
+  uint32_t ck_pos = 0, ck_end = 0;  // this warp's claimed run of issue positions [ck_pos, ck_end)
   while (true) {
     // work item: a queued split subtask first (Alg 4 L3-4), else the next root (Alg 4 L6, heaviest =
     // highest rank first); both end in the single dispatch site below
+    uint32_t task = kNone;
+    if (lane == 0) task = queue_pop(P);  // split subtasks first (Alg 4 L3), also inside a root chunk
+    task = __shfl_sync(GMBE_FULL, task, 0);
+    if (task == kNone && roots_done) {
+      // 3. idle: all roots issued -- wait for a task or for termination (nothing queued or running)
+      unsigned long long pend = 0;
+      if (lane == 0) pend = ld_volatile(&P.ctrl->pending.v);
+      pend = __shfl_sync(GMBE_FULL, pend, 0);
+      if (pend == 0) break;
+      if (!is_hungry && P.donate) {  // ask the working warps to donate (see donate_reg)
+        if (lane == 0) atomicAdd(&P.ctrl->hungry.v, 1ull);
+        is_hungry = true;
+      }
+      __nanosleep(idle < 4 ? 500 : (idle < 16 ? 2000 : 8000));  // exponential-ish backoff
+      idle++;
+      continue;
+    }
+    WarpMem M = GMBE_WARP_MEM();
     TaskCtx Tc;
     uint32_t* top = nullptr;
     uint32_t* lo = M.dyn;
     uint32_t lmap = 0, kind = 2, item = 0, tl_l = 0, tl_c = 0;
     const long long c0 = P.per_root_cycles ? clock64() : 0;
     const unsigned long long g0 = P.timeline ? globaltimer() : 0, n0 = P.timeline ? A.get(kAcNodes) : 0ull;
-    uint32_t task = kNone;
-    if (lane == 0) task = queue_pop(P);  // split subtasks first (Alg 4 L3), also inside a root chunk
-    task = __shfl_sync(GMBE_FULL, task, 0);
     bool release = true;  // this item ends a unit of `pending` (a task, or a chunk's last root)
     if (task != kNone) {
       if (is_hungry) {
@@ -2581,11 +2630,11 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
       item = Tc.root;
       tl_l = top[2];
       tl_c = top[0];
-    } else if (!roots_done) {
+    } else {
       if (ck_pos == ck_end) {
-        // claim a chunk of consecutive issue positions with ONE atomic: single roots in the heavy
-        // head of the issue list, P.chunk roots once this warp has seen positions past
-        // P.chunk_from (the estimate may be stale; any K gives disjoint ranges)
+        // claim a run of consecutive issue positions with ONE atomic: single roots in the heavy head
+        // of the issue list, P.chunk roots once this warp has seen positions past P.chunk_from (the
+        // estimate may be stale; any run length gives disjoint ranges)
         const uint32_t K = ck_end >= P.chunk_from ? P.chunk : 1u;
         unsigned long long t = 0;
         if (lane == 0) {
@@ -2598,61 +2647,36 @@ __global__ void __launch_bounds__(32 * GMBE_WPB, GMBE_MIN_BLOCKS) k_enum(const P
         if (t < P.n_roots) {
           ck_pos = (uint32_t)t;
           ck_end = (uint32_t)min(t + K, (unsigned long long)P.n_roots);
-          ck_base = ck_pos;
-          // prefetch the chunk: lane j holds the root at position ck_base + j and its N(v) range
-          const uint32_t q = ck_pos + lane;
-          ck_rk = q < ck_end ? P.issue[q] : 0u;
-          ck_lb = q < ck_end ? P.g.off_v[ck_rk] : 0u;
-          ck_l = q < ck_end ? P.g.off_v[ck_rk + 1] - ck_lb : 0u;
         } else {
           if (lane == 0) atomicAdd(&P.ctrl->pending.v, ~0ull);
           roots_done = true;
+          continue;
         }
       }
-      if (!roots_done) {
-        const uint32_t jq = ck_pos - ck_base;
-        const uint32_t rk = __shfl_sync(GMBE_FULL, ck_rk, jq);
-        const uint32_t rlb = __shfl_sync(GMBE_FULL, ck_lb, jq), rl = __shfl_sync(GMBE_FULL, ck_l, jq);
-        ck_pos++;
-        release = ck_pos == ck_end;
-        kind = 0;
-        item = rk;
-        if (run_root(P, rk, rlb, rl, M, A, Tc, &top, &lo)) lmap = top[2];
-        if (P.debug & 1024) top = nullptr;  // experiments: root construction only (no subtrees)
-        tl_l = rl;
-      }
+      const uint32_t rk = P.issue[ck_pos];
+      const uint32_t rlb = P.g.off_v[rk], rl = P.g.off_v[rk + 1] - rlb;
+      ck_pos++;
+      release = ck_pos == ck_end;
+      kind = 0;
+      item = rk;
+      if (run_root(P, rk, rlb, rl, M, A, Tc, &top, &lo)) lmap = top[2];
+      if (P.debug & 1024) top = nullptr;  // experiments: root construction only (no subtrees)
+      tl_l = rl;
     }
-    if (kind != 2) {
-      if (top) dispatch_task(P, Tc, top, lo, M.dyn_end, lmap, A, M.sm_sort, &s_thr[threadIdx.x >> 5]);
-      if (P.timeline) timeline_rec(P, kind, item, g0, tl_info(A.get(kAcNodes) - n0, tl_l, tl_c));
-      if (P.per_root_cycles && lane == 0)
-        atomicAdd(P.per_root_cycles + item, (unsigned long long)(clock64() - c0));
-      __syncwarp();
-      if (lane == 0 && release) atomicAdd(&P.ctrl->pending.v, ~0ull);
-      idle = 0;
-      continue;
-    }
-    if (!roots_done) continue;
-    // 3. termination: all roots issued and nothing queued or running
-    unsigned long long pend = 0;
-    if (lane == 0) pend = ld_volatile(&P.ctrl->pending.v);
-    pend = __shfl_sync(GMBE_FULL, pend, 0);
-    if (pend == 0) break;
-    if (!is_hungry && P.donate) {  // ask the working warps to donate (see donate_reg)
-      if (lane == 0) atomicAdd(&P.ctrl->hungry.v, 1ull);
-      is_hungry = true;
-    }
-    __nanosleep(idle < 4 ? 500 : (idle < 16 ? 2000 : 8000));  // exponential-ish backoff
-    idle++;
+    if (top) dispatch_task(P, Tc, top, lo, M.dyn_end, lmap, A, M.sm_sort, &s_thr[threadIdx.x >> 5]);
+    if (P.timeline) timeline_rec(P, kind, item, g0, tl_info(A.get(kAcNodes) - n0, tl_l, tl_c));
+    if (P.per_root_cycles && lane == 0)
+      atomicAdd(P.per_root_cycles + item, (unsigned long long)(clock64() - c0));
+    __syncwarp();
+    if (lane == 0 && release) atomicAdd(&P.ctrl->pending.v, ~0ull);
+    idle = 0;
   }
+#undef GMBE_WARP_MEM
   if (lane < kAcN) atomicAdd(&P.ctrl->count + lane, A.v);  // Ctrl's counters, in kAc* order
-  if (lane == 0) {
-    Ctrl* c = P.ctrl;
 #ifdef GMBE_PROFILE
-    if (P.profile)
-      for (int k = 0; k < 16; k++) atomicAdd(&c->phase[k], A.ph[k]);
+  if (lane == 0 && P.profile)
+    for (int k = 0; k < 16; k++) atomicAdd(&P.ctrl->phase[k], A.ph[k]);
 #endif
-  }
 }
 
 #include "gmbe_block.cuh"  // GMBE-BLOCK (block-centric ablation variant)

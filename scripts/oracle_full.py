@@ -48,6 +48,8 @@ def main():
     ap.add_argument("config")
     ap.add_argument("--procs", type=int, default=len(os.sched_getaffinity(0)))
     ap.add_argument("--shards", type=int, default=0, help="root shards (default 4 x procs)")
+    ap.add_argument("--outdir", default=os.path.join(ROOT, "profiles"))
+    ap.add_argument("--tag", default="", help="suffix of the output names (e.g. _box)")
     a = ap.parse_args()
     import oracle
     oracle.build()
@@ -67,10 +69,10 @@ def main():
            "cpu_model": _cpu_model(), "host_cores": os.cpu_count(),
            "rate_per_core": count / (float(ns.sum()) * 1e-9),
            "rate_all_procs": count / wall}
-    os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
-    with open(os.path.join(ROOT, "profiles", "oracle_full_%s.json" % a.config), "w") as f:
+    os.makedirs(a.outdir, exist_ok=True)
+    with open(os.path.join(a.outdir, "oracle_full_%s%s.json" % (a.config, a.tag)), "w") as f:
         json.dump(out, f, indent=1)
-    np.savez_compressed(os.path.join(ROOT, "profiles", "oracle_roots_%s.npz" % a.config), ns=ns, count=cnt)
+    np.savez_compressed(os.path.join(a.outdir, "oracle_roots_%s%s.npz" % (a.config, a.tag)), ns=ns, count=cnt)
     print(json.dumps(out))
 
 
