@@ -1635,10 +1635,6 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
   ThrLevel stk[32];
   bool has = lane == 0;
   unsigned long long L = L0, SR = ((unsigned long long)rec[7] << 32) | rec[6];
-  // SL = Σ_{u∈L} hU(u) of the lane's current node, kept incrementally (children subtract the members
-  // they drop, pops add them back), so the maximality loop can stop as soon as L' is proven maximal
-  unsigned long long SL = 0;
-  for (unsigned long long m = L0; m; m &= m - 1) SL += cols[__ffsll(m) - 1].hu;
   const uint32_t cand_all = nC >= 32 ? GMBE_FULL : ((1u << nC) - 1u);
   uint32_t C = cand_all, next = 0, Rm = 0, d = 0, dmask = 0;
   uint32_t bd = 0;  // tree depth (below the job's top) of this lane's level 0
@@ -1662,9 +1658,7 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
         const uint32_t rmp = stk[d].Rm, diff = Rm & ~rmp;  // {i} ∪ absorbed of the finished child
         next = __ffs(diff);
         for (uint32_t m = diff; m; m &= m - 1) SR -= ts->hv[__ffs(m) - 1];
-        const unsigned long long lpar = stk[d].L;
-        for (unsigned long long m = lpar & ~L; m; m &= m - 1) SL += cols[__ffsll(m) - 1].hu;
-        L = lpar;
+        L = stk[d].L;
         C = stk[d].C;
         Rm = rmp;
         dmask &= ~(1u << d);
@@ -1738,8 +1732,6 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
           bd = (uint32_t)(o[3] >> 32);
           d = 0;
           dmask = 0;
-          SL = 0;
-          for (unsigned long long m = L; m; m &= m - 1) SL += cols[__ffsll(m) - 1].hu;
         }
         __syncwarp();  // the slots are read before any donor of a later step rewrites them
       }
@@ -1787,20 +1779,22 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
       sl = cols[j].hu;
     } else {  // |L'| >= 2: no Q pattern and no job candidate outside R' may cover L'
       const uint32_t outside = cand_all & ~(Rm | (1u << i) | ab);
-      unsigned long long qa = ~0ull;
+      unsigned long long qa = ~0ull, m = lp;
       uint32_t ca = GMBE_FULL;
-      for (unsigned long long m = lp; m; m &= m - 1) {
+      for (; m; m &= m - 1) {
         const uint32_t j = __ffsll(m) - 1;
-        qa &= cols[j].q;
+        const ThrCol tc = cols[j];
+        qa &= tc.q;
+        sl += tc.hu;
         ca &= ts->ccol[j];
-        if (!qa && !(ca & outside)) break;
+        if (!qa && !(ca & outside)) {
+          m &= m - 1;
+          break;
+        }
       }
       maximal = !qa && !(ca & outside);
-      // SL(L') from the node's SL(L): remove the members L' dropped (usually a few)
-      if (maximal) {
-        sl = SL;
-        for (unsigned long long m = L & ~lp; m; m &= m - 1) sl -= cols[__ffsll(m) - 1].hu;
-      }
+      if (maximal)
+        for (; m; m &= m - 1) sl += cols[__ffsll(m) - 1].hu;
     }
     if (!maximal) {
       n_nonmax++;
@@ -1825,7 +1819,6 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
     d++;
     L = lp;
     SR = srn;
-    SL = sl;
     C = cd;
     Rm = rmn;
     next = 0;
@@ -1911,6 +1904,37 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     int r;
     if constexpr (SMALL) r = gen_child_small(P, T, cur, i, ch, A, smem);
     else r = gen_child(P, T, cur, i, ch, A, smem, lpe);
+    // dynamic donation at the warp level (as donate_reg / donate_thr do in the tiers below): while
+    // other warps are idle, the remaining children of cur -- its candidates after i, already
+    // compacted by this child's Thm 4.1 pass -- go to the queue as one subtask (node (L, R, SR of cur,
+    // those candidates)); its children, later sets and prune marks are the ones this warp would have
+    // generated, so the tree and every counter are unchanged
+    if (P.donate && !(split_mode && cur == top) && cur[0] >= i + 3 && hungry(P)) {
+      uint32_t* scr = align4(ch + (r == 2 ? rec_words(T, ch) : 0));
+      const uint32_t n = cur[0] - (i + 1);
+      const uint32_t words = kHdr + T.W4 + n * T.E;
+      if (scr + words <= stack_hi) {
+        const uint32_t* src = cur + kHdr + T.W4 + (size_t)(i + 1) * T.E;
+        for (uint32_t j = lane; j < T.W4; j += 32) scr[kHdr + j] = cur[kHdr + j];
+        for (uint32_t j = lane; j < n * T.E; j += 32) scr[kHdr + T.W4 + j] = src[j];
+        if (lane == 0) {
+          scr[0] = n;
+          scr[1] = 0;
+          scr[2] = cur[2];
+          scr[3] = 0;
+          scr[4] = kNone;
+          scr[5] = cur[5];
+          scr[6] = cur[6];
+          scr[7] = cur[7];
+        }
+        __syncwarp();
+        if (task_publish(P, T, lmap, T.rlist ? cur[5] : 0, scr, words, A)) {
+          A.add(kAcDonations, 1);
+          if (lane == 0) cur[0] = i + 1;  // cur's remaining children now belong to the subtask
+          __syncwarp();
+        }
+      }
+    }
     // Alg 4 L25: hand the child to the task queue as a self-contained subtask -- every child of a
     // heavy top, and (wide universes) any child that is itself heavy (reading B4)
     if (r == 2 && ((split_mode && cur == top) || (!SMALL && heavy_wide(P, lmap, ch[0])))) {
