@@ -75,15 +75,48 @@ def _peaks():
         return 6650.0, "fallback"
 
 
-def _traffic(name):
-    """DRAM bytes per k_enum launch from the committed ncu --set full summary, if any."""
+def _ncu(name):
+    """The committed ncu --set full summary of k_enum on this config (profiles/ncu_summary.json)."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         with open(p) as f:
-            d = json.load(f)
-        return d[name]["dram_bytes_per_launch"]
+            return json.load(f).get(name)
     except Exception:
         return None
+
+
+def _traffic(name):
+    """DRAM bytes per k_enum launch from the committed ncu --set full summary, if any."""
+    d = _ncu(name)
+    return d.get("dram_bytes_per_launch") if d else None
+
+
+def _secondary(name, peak_hbm):
+    """Secondary rooflines of k_enum from the committed ncu capture: L2 bytes against the measured L2
+    read peak (profiles/r02_l2_peak.json, scripts/l2peak.cu), issued warp instructions against the
+    SM issue peak (148 SMs x 4 schedulers x 1 warp-instruction/clock at the capture's SM clock)."""
+    d = _ncu(name)
+    if not d or not d.get("kernel_ms_under_ncu"):
+        return None
+    out = {"source": d.get("source")}
+    t = d["kernel_ms_under_ncu"] * 1e-3
+    try:
+        with open(os.path.join(ROOT, "profiles", "r02_l2_peak.json")) as f:
+            l2 = json.load(f)["l2_read_gbs"]
+        if d.get("l2_bytes_per_launch"):
+            a = d["l2_bytes_per_launch"] / t / 1e9
+            out["l2"] = {"achieved": a, "peak": l2, "unit": "GB/s", "frac": a / l2, "peak_kind": "measured (l2peak.cu)"}
+    except Exception:
+        pass
+    if d.get("warp_inst_per_launch") and d.get("sm_mhz"):
+        a = d["warp_inst_per_launch"] / t / 1e9
+        pk = 148 * 4 * d["sm_mhz"] * 1e6 / 1e9
+        out["issue"] = {"achieved": a, "peak": pk, "unit": "G warp-inst/s", "frac": a / pk,
+                        "warp_execution_efficiency": d.get("warp_execution_efficiency")}
+    if d.get("dram_bytes_per_launch"):
+        a = d["dram_bytes_per_launch"] / t / 1e9
+        out["dram"] = {"achieved": a, "peak": peak_hbm, "unit": "GB/s", "frac": a / peak_hbm}
+    return out
 
 
 def _profile(name):
@@ -440,7 +473,12 @@ def main():
                          "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": _traffic(a.config),
                          "algo_bytes_per_launch": abytes, "algo_bytes_definition": adef,
-                         "algo_bytes_cand": ab_rank},
+                         "algo_bytes_cand": ab_rank,
+                         # the bytes the kernel itself streams (wedge + candidate terms, counted on
+                         # the device): the filtered-Q term of the survey's numerator is replaced by
+                         # Γ-index tests in this kernel, so this is the stricter fraction
+                         "frac_cand": (ab_rank / (k_rank * 1e-3) / 1e9) / peak if k_rank > 0 else 0.0,
+                         "secondary": _secondary(a.config, peak)},
             "work": {"nodes": rc.nodes, "nonmax": rc.nonmax, "roots_run": rc.roots_run,
                      "splits": rc.splits, "tasks": rc.tasks, "donations": rc.donations},
             "clocks": clocks,

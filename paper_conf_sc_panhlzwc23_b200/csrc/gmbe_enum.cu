@@ -1494,6 +1494,9 @@ __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const
 #ifndef GMBE_ROOT_CHUNK
 #define GMBE_ROOT_CHUNK 1  // light roots claimed per atomic (opts.root_chunk); >1 measured slower on the heavy-tailed shapes
 #endif
+#ifndef GMBE_THR_DONATE_BURST
+#define GMBE_THR_DONATE_BURST 4  // run_thr: levels donated per check while other warps are hungry
+#endif
 #ifndef GMBE_THR_MIN_EST
 #define GMBE_THR_MIN_EST 16  // jobs with fewer adjacency bits (Σ(k-1)) stay on run_reg (setup > work)
 #endif
@@ -1672,12 +1675,14 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
       want = __shfl_sync(GMBE_FULL, hflag, 0) != 0 || (P.debug & 8);
       if (lane == 0) hflag = ld_volatile(&P.ctrl->hungry.v) != 0;  // latency hidden until the next check
     }
-    if (want) {  // cross-warp donation to idle warps
+    // cross-warp donation to idle warps: up to GMBE_THR_DONATE_BURST levels per check
+    for (uint32_t burst = 0; want && burst < GMBE_THR_DONATE_BURST; burst++) {
       // the donor: the lane whose shallowest stacked level with untraversed children is the
       // shallowest in the job's tree (the largest piece of remaining work)
       const uint32_t key =
           __reduce_min_sync(GMBE_FULL, dmask ? ((bd + (uint32_t)(__ffs(dmask) - 1)) << 5) | lane : kNone);
-      if (key != kNone) {
+      want = key != kNone;
+      if (want) {
         const uint32_t src = key & 31u;
         const uint32_t k = lane == src ? (uint32_t)(__ffs(dmask) - 1) : 0u;
         unsigned long long kL = 0, kSR = 0;
@@ -1690,11 +1695,12 @@ __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& 
           kSR = SR;
           for (uint32_t m = Rm & ~kRm; m; m &= m - 1) kSR -= ts->hv[__ffs(m) - 1];
         }
-        if (donate_thr(P, T, lmap, A, ts, nC, rlen0, src, kL, kSR, kC, kRm, knext, scratch, scratch_end) &&
-            lane == src) {
+        const bool ok = donate_thr(P, T, lmap, A, ts, nC, rlen0, src, kL, kSR, kC, kRm, knext, scratch, scratch_end);
+        if (ok && lane == src) {
           stk[k].C &= knext >= 32 ? GMBE_FULL : (1u << knext) - 1u;  // its remaining children left
           dmask &= ~(1u << k);
         }
+        want = ok;
       }
     }
 #endif

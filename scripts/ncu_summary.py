@@ -35,6 +35,12 @@ try:  # derived: achieved L2 and DRAM bandwidth, warp execution efficiency
     dr = sum(float(m[k][0].replace(",", "")) * mult[m[k][1].strip()] for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
     summ["derived_dram_GBps"] = round(dr / t_s / 1e9, 1)
     summ["derived_warp_execution_efficiency"] = round(float(m["smsp__thread_inst_executed_per_inst_executed.ratio"][0]) / 32, 3)
+    # the per-launch fields bench.py's roofline reads (profiles/ncu_summary.json)
+    summ["per_launch"] = {
+        "kernel_ms_under_ncu": t_s * 1e3, "dram_bytes_per_launch": int(dr), "l2_bytes_per_launch": int(l2),
+        "warp_inst_per_launch": int(float(m["smsp__inst_executed.sum"][0].replace(",", ""))),
+        "sm_mhz": round(float(m["sm__cycles_active.avg"][0].replace(",", "")) / t_s / 1e6, 1),
+        "warp_execution_efficiency": summ["derived_warp_execution_efficiency"]}
 except (KeyError, ValueError):
     pass
 st = {h[len("smsp__pcsamp_warps_issue_stalled_"):]: float(v.replace(",", "") or 0) for h, (v, u) in m.items()
