@@ -268,19 +268,12 @@ __device__ __forceinline__ uint32_t ht_insert_warp(uint32_t* keys, uint32_t shif
   while (__any_sync(GMBE_FULL, pend)) {
     bool ins = false;
     if (pend) {
-      const uint32_t k = ldv(keys + h);
-      if (k == v) {
+      // one round trip per probe: a CAS on a slot that already holds v just returns v
+      const uint32_t old = atomicCAS(keys + h, GMBE_EMPTY, v);
+      if (old == GMBE_EMPTY || old == v) {
         slot = h;
         pend = false;
-      } else if (k == GMBE_EMPTY) {
-        const uint32_t old = atomicCAS(keys + h, GMBE_EMPTY, v);
-        if (old == GMBE_EMPTY || old == v) {
-          slot = h;
-          pend = false;
-          ins = old == GMBE_EMPTY;
-        } else {
-          h = (h + 1) & mask;
-        }
+        ins = old == GMBE_EMPTY;
       } else {
         h = (h + 1) & mask;
       }
@@ -1495,7 +1488,7 @@ __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const
 #define GMBE_ROOT_CHUNK 1  // light roots claimed per atomic (opts.root_chunk); >1 measured slower on the heavy-tailed shapes
 #endif
 #ifndef GMBE_THR_DONATE_BURST
-#define GMBE_THR_DONATE_BURST 4  // run_thr: levels donated per check while other warps are hungry
+#define GMBE_THR_DONATE_BURST 1  // run_thr: levels donated per check while other warps are hungry (4, 16 measured no better)
 #endif
 #ifndef GMBE_THR_MIN_EST
 #define GMBE_THR_MIN_EST 16  // jobs with fewer adjacency bits (Σ(k-1)) stay on run_reg (setup > work)

@@ -2,6 +2,7 @@
 # round 2 evidence: bench lines (all shapes), reference arm, launch list, ncu full of k_enum, Fig 9
 cd "${GRAFT_REPO_ROOT:-.}"; mkdir -p gpurun_out
 nvidia-smi --query-gpu=clocks.sm,clocks.max.sm --format=csv > gpurun_out/ev_clocks.txt
+[ -x scripts/l2peak ] || nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o scripts/l2peak scripts/l2peak.cu
 ./scripts/l2peak > gpurun_out/ev_l2peak.txt 2>&1
 timeout 900 python bench.py > gpurun_out/ev_bench_gh_work.json 2> gpurun_out/ev_bench_gh_work.err
 for c in dblp bx bx_work yg_work gh yg; do
@@ -15,3 +16,5 @@ python scripts/ncu_summary.py gpurun_out/ev_gh_work.ncu-rep --json gpurun_out/ev
 for c in gh_work bx_work; do timeout 900 python scripts/fig9_sched.py $c --out gpurun_out/ev_fig9_$c.json > gpurun_out/ev_fig9_$c.log 2>&1; done
 for f in gpurun_out/ev_bench_*.json; do echo "== $f"; cat $f | cut -c1-400; done
 cat gpurun_out/ev_launches_gh_work.txt | head -12; cat gpurun_out/ev_ncu_gh_work.txt | head -24; tail -2 gpurun_out/ev_fig9_*.log
+for c in gh_work bx_work dblp; do timeout 900 python scripts/shard_times.py $c 2 4 8 mode=cost > gpurun_out/ev_shards_$c.json 2>&1; done
+cat gpurun_out/ev_shards_*.json | cut -c1-600
