@@ -2713,6 +2713,7 @@ struct Workspace {
   bool clean = false;
   uint64_t tmax = 0, omax = 0, bmax = 0, dyn = 0, nwarps = 0, pool_auto = 0;  // cached sizing
   bool dyn_capped = false;
+  bool dyn_failed = false;  // an arena allocation of the free-memory-derived size failed (halved)
   int sms = 0, bps_max = 0, bps_max_blk = 0;
   void* pool = nullptr;
   size_t pool_bytes = 0;
@@ -2886,7 +2887,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   uint64_t arena_words;
   bool reuse = W.arena && W.nwarps == nwarps && W.tmax >= tmax && W.omax >= omax && W.bmax >= bmax &&
                (W.dyn >= dyn_want || (!o.arena_words && W.dyn_capped));
-  if (reuse && W.dyn < dyn_want) {
+  if (reuse && W.dyn < dyn_want && !W.dyn_failed) {
     // a layout capped by free memory at an earlier call: re-size if there is more room now
     size_t fr = 0, tot = 0;
     GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
@@ -2894,7 +2895,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
     const uint64_t fixed = 3 * W.tmax + W.bmax + W.omax + 8;
     const uint64_t cap_total = (uint64_t)(fr * 0.5) / 4 / nwarps;
     const uint64_t cap_now = cap_total > fixed ? cap_total - fixed : 0;
-    if (cap_now > W.dyn + W.dyn / 8) reuse = false;
+    if (cap_now > W.dyn + W.dyn / 2) reuse = false;  // (hysteresis: re-size only for a real gain)
   }
   uint64_t bmax_use = bmax;
   if (reuse) {
@@ -2950,6 +2951,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
       (void)cudaGetLastError();
       W.dyn = std::max<uint64_t>(W.dyn / 2, 1u << 16);
       W.dyn_capped = true;
+      W.dyn_failed = true;  // do not try to grow again on later calls (gmbe_release_workspace resets)
       arena_words = (3 * tmax + bmax_use + omax + 8 + W.dyn + 3) & ~3ull;
       ae = ensure(&W.arena, &W.arena_bytes, nwarps * arena_words * 4);
     }
