@@ -2714,6 +2714,7 @@ struct Workspace {
   uint64_t tmax = 0, omax = 0, bmax = 0, dyn = 0, nwarps = 0, pool_auto = 0;  // cached sizing
   bool dyn_capped = false;
   bool dyn_failed = false;  // an arena allocation of the free-memory-derived size failed (halved)
+  bool regrow = false;      // the last call ran out of a capped arena: re-check free memory once
   int sms = 0, bps_max = 0, bps_max_blk = 0;
   void* pool = nullptr;
   size_t pool_bytes = 0;
@@ -2887,7 +2888,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   uint64_t arena_words;
   bool reuse = W.arena && W.nwarps == nwarps && W.tmax >= tmax && W.omax >= omax && W.bmax >= bmax &&
                (W.dyn >= dyn_want || (!o.arena_words && W.dyn_capped));
-  if (reuse && W.dyn < dyn_want && !W.dyn_failed) {
+  if (reuse && W.dyn < dyn_want && W.regrow && !W.dyn_failed) {
     // a layout capped by free memory at an earlier call: re-size if there is more room now
     size_t fr = 0, tot = 0;
     GMBE_CUDA_TRY(cudaMemGetInfo(&fr, &tot));
@@ -2897,6 +2898,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
     const uint64_t cap_now = cap_total > fixed ? cap_total - fixed : 0;
     if (cap_now > W.dyn + W.dyn / 2) reuse = false;  // (hysteresis: re-size only for a real gain)
   }
+  W.regrow = false;
   uint64_t bmax_use = bmax;
   if (reuse) {
     tmax = W.tmax;
@@ -3180,6 +3182,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   }
   if (hc.error) {
     W.clean = false;
+    W.regrow = W.dyn_capped;  // a capped arena was too small: the next call re-checks free memory
     return gmbe_set_error(GMBE_EINTERNAL,
                           "gmbe_enumerate: per-warp workspace exceeded; raise opts.arena_words");
   }
