@@ -127,7 +127,8 @@ typedef struct {
    * subtask, 2 split descriptor) -- the active-SM timeline of PAPER.md Fig 4 / Fig 9. */
   uint64_t* timeline;
   uint64_t timeline_cap;
-  /* Workspace (0 = auto): words of the per-warp dynamic region (root record, node stack); words
+  /* Workspace (0 = auto): words of the per-warp dynamic region (root record, node stack; a caller-given
+   * size is the first attempt's, see gmbe_result.retries); words
    * of the task pool (split subtasks and shared Γ columns; when it is exhausted work simply stays
    * with the warp that generated it); capacity of the task queue (entries). */
   uint64_t arena_words;
@@ -183,12 +184,17 @@ typedef struct {
   uint64_t splits;        /* nodes expanded in split mode */
   uint64_t tasks;         /* subtasks enqueued */
   uint64_t donations;     /* subtasks donated to idle warps (dynamic load balancing) */
-  double kernel_ms;       /* device time of the enumeration kernel (CUDA events) */
+  double kernel_ms;       /* device time of the enumeration kernel (CUDA events; the last run) */
+  uint64_t retries;       /* re-runs after a per-warp workspace overflow (degrade path: larger per-warp
+                             regions -- a caller-given arena_words is replaced by the automatic size, an
+                             automatic size goes to fewer resident warps, 24 -> 16 -> 8 per SM; not for
+                             streaming calls) */
 } gmbe_result;
 
 /* Enumerate all maximal bicliques of g (or of one root shard).  Synchronous: returns after the
  * result is on the host.  Concurrent calls on one graph must use distinct streams.
- * Errors: EINVAL (NULL g/out, part_index >= part_count), ENOMEM, ECUDA, EINTERNAL. */
+ * Errors: EINVAL (NULL g/out, part_index >= part_count), ENOMEM, ECUDA, EINTERNAL (a per-warp workspace
+ * still overflowed after the degrade path's re-runs). */
 int gmbe_enumerate(const gmbe_graph* g, const gmbe_opts* opts, gmbe_result* out);
 
 /* Streaming output (the problem statement asks to *enumerate* all maximal

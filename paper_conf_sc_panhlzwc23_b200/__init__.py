@@ -64,7 +64,7 @@ class Opts(ctypes.Structure):
 class CResult(ctypes.Structure):
     _fields_ = [(n, _u64) for n in ("count", "checksum", "n_written", "truncated", "roots_run",
                                      "nodes", "nonmax", "algo_bytes_cand", "splits",
-                                     "tasks", "donations")] + [("kernel_ms", ctypes.c_double)]
+                                     "tasks", "donations")] + [("kernel_ms", ctypes.c_double), ("retries", _u64)]
 
 
 _lib.gmbe_load_bipartite.argtypes = [_u32, _u32, _vp, _u64, ctypes.POINTER(LoadOpts), ctypes.POINTER(_vp)]
@@ -138,6 +138,7 @@ class Result:
     tasks: int
     donations: int
     kernel_ms: float
+    retries: int = 0
     bicliques: list = field(default=None, repr=False)
     per_root_count: np.ndarray = field(default=None, repr=False)
     per_root_cycles: np.ndarray = field(default=None, repr=False)

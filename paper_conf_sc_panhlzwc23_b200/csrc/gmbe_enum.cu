@@ -2830,6 +2830,16 @@ extern "C" int gmbe_enumerate_stream(const gmbe_graph* G, const gmbe_opts* opts,
   return enumerate_impl(G, opts, sink, user, ring_words, out);
 }
 
+static int enumerate_once(const gmbe_graph* G, const gmbe_opts& o, gmbe_sink_fn sink, void* user,
+                          uint64_t ring_words, gmbe_result* out, bool* arena_overflow);
+
+// Degrade path for a per-warp workspace overflow (a root record or a DFS level that does not fit the
+// warp's dynamic region): the call is re-run from scratch with larger per-warp regions -- a caller-given
+// arena_words is replaced by the automatic size (the full bound, capped by free memory), an automatic
+// size is spread over fewer resident warps (24 -> 16 -> 8 per SM, the free-memory cap being shared by
+// fewer warps).  The kernel writes nothing the
+// caller sees until it completes (counters, bounded records), so the re-run is exact; a streaming call
+// (records already delivered) is not re-run.
 static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_fn sink, void* user,
                           uint64_t ring_words, gmbe_result* out) {
   if (!G || !out) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: NULL argument");
@@ -2838,6 +2848,23 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
     if (opts->struct_size > sizeof(gmbe_opts)) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: bad struct_size");
     std::memcpy(&o, opts, opts->struct_size);
   }
+  for (uint32_t attempt = 0;; attempt++) {
+    bool ovf = false;
+    const int rc = enumerate_once(G, o, sink, user, ring_words, out, &ovf);
+    if (rc == GMBE_OK) out->retries = attempt;
+    if (rc == GMBE_OK || !ovf || sink || attempt >= 6) return rc;
+    if (o.arena_words) {
+      o.arena_words = 0;  // the automatic size: the full bound, capped by free memory
+    } else {
+      const uint32_t wps = o.warps_per_sm ? std::min<uint32_t>(o.warps_per_sm, 24u) : 24u;
+      if (wps <= kWpb) return rc;
+      o.warps_per_sm = wps > 16 ? 16 : kWpb;
+    }
+  }
+}
+
+static int enumerate_once(const gmbe_graph* G, const gmbe_opts& o, gmbe_sink_fn sink, void* user,
+                          uint64_t ring_words, gmbe_result* out, bool* arena_overflow) {
   const uint32_t parts = o.part_count ? o.part_count : 1;
   if (o.part_index >= parts) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: part_index >= part_count");
   if (o.part_mode > GMBE_PART_COST) return gmbe_set_error(GMBE_EINVAL, "gmbe_enumerate: bad part_mode");
@@ -3183,6 +3210,7 @@ static int enumerate_impl(const gmbe_graph* G, const gmbe_opts* opts, gmbe_sink_
   if (hc.error) {
     W.clean = false;
     W.regrow = W.dyn_capped;  // a capped arena was too small: the next call re-checks free memory
+    *arena_overflow = true;
     return gmbe_set_error(GMBE_EINTERNAL,
                           "gmbe_enumerate: per-warp workspace exceeded; raise opts.arena_words");
   }

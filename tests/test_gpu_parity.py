@@ -848,3 +848,24 @@ def test_root_chunk_invariance(gmbe, dense_case):
             assert (r.count, r.checksum, r.nodes) == (gd["count"], int(gd["checksum"], 16), gd["nodes"])
     finally:
         g.free()
+
+
+# ---------------------------------------------------------------- arena overflow degrade path
+@pytest.mark.parametrize("name", ["gh", "bx"])
+def test_arena_overflow_degrade_path(gmbe, name):
+    """A per-warp dynamic region far too small for the graph's root records (arena_words=4096) no
+    longer fails the call: it is re-run with 4x larger regions until it fits (result.retries > 0),
+    and the result is the golden's, bit-exact.  The next call with the default sizing needs no
+    re-run."""
+    gd = _gold_cfg()[name]
+    nu, nv, e = make_config(name)
+    g = gmbe.load(nu, nv, e)
+    try:
+        r = g.enumerate(arena_words=4096)
+        assert r.retries > 0
+        assert (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16))
+        assert (r.nodes, r.nonmax, r.roots_run) == (gd["nodes"], gd["nonmax"], gd["roots_run"])
+        r = g.enumerate()
+        assert r.retries == 0 and (r.count, r.checksum) == (gd["count"], int(gd["checksum"], 16))
+    finally:
+        g.free()
