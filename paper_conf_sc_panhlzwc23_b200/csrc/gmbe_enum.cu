@@ -730,43 +730,23 @@ __device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_is_r(const Params& P, const uint
   const uint32_t* n0 = g.adj_u + g.off_u[u0];
   uint32_t count = 0;
   if (lc > 32) {
-    // wide L', two phases.  A (lane per vertex): 32 vertices of N(u*) at a time go through the first
-    // kFilter members of L' (scratch order) -- a vertex outside Γ(L') almost always fails one of
-    // them, so most of N(u*) costs a few lane-parallel binary searches instead of a sequential one
-    // per vertex.  B: each survivor is tested against every member, 32 members per step (a member of
-    // Γ(L') -- every vertex of R' -- costs ⌈|L'|/32⌉ steps).
-    constexpr uint32_t kFilter = 8;
-    const uint32_t nf = lc < kFilter ? lc : kFilter;
-    uint32_t fb = 0, fd = 0;  // lane t < nf: (begin, degree) of filter member t
-    if (lane < nf) {
-      const unsigned long long kt = scratch[lane];
-      fb = g.off_u[(uint32_t)kt];
-      fd = (uint32_t)(kt >> 32);
-    }
-    for (uint32_t b = 0; b < d0; b += 32) {
-      const uint32_t idx = b + lane;
-      bool ok = idx < d0;
-      const uint32_t v = ok ? __ldg(n0 + idx) : 0u;
-      for (uint32_t t = 0; t < nf && __any_sync(GMBE_FULL, ok); t++) {
-        const uint32_t jb = __shfl_sync(GMBE_FULL, fb, t), jd = __shfl_sync(GMBE_FULL, fd, t);
-        if (ok) ok = bsearch_rank(g.adj_u + jb, jd, v);
-      }
-      for (uint32_t surv = __ballot_sync(GMBE_FULL, ok); surv; surv &= surv - 1) {
-        const uint32_t vv = __shfl_sync(GMBE_FULL, v, __ffs(surv) - 1);
-        bool all = true;
-        for (uint32_t j0 = 0; j0 < lc && all; j0 += 32) {  // (u* itself passes trivially)
-          const uint32_t j = j0 + lane;
-          bool in = true;
-          if (j < lc) {
-            const unsigned long long kj = scratch[j];
-            const uint32_t jb = g.off_u[(uint32_t)kj];
-            in = bsearch_rank(g.adj_u + jb, (uint32_t)(kj >> 32), vv);
-          }
-          all = __all_sync(GMBE_FULL, in);
+    // wide L': one v ∈ N(u*) at a time, lanes test 32 members per step (a member of Γ(L') -- every
+    // vertex of R' -- costs ⌈|L'|/32⌉ steps instead of |L'| - 1; others usually fail in the first)
+    for (uint32_t b = 0; b < d0; b++) {
+      const uint32_t v = __ldg(n0 + b);
+      bool all = true;
+      for (uint32_t j0 = 0; j0 < lc && all; j0 += 32) {  // (u* itself passes trivially)
+        const uint32_t j = j0 + lane;
+        bool in = true;
+        if (j < lc) {
+          const unsigned long long kj = scratch[j];
+          const uint32_t jb = g.off_u[(uint32_t)kj];
+          in = bsearch_rank(g.adj_u + jb, (uint32_t)(kj >> 32), v);
         }
-        count += all;
-        if (count > rlen) return false;
+        all = __all_sync(GMBE_FULL, in);
       }
+      count += all;
+      if (count > rlen) return false;
     }
     return count == rlen;
   }
