@@ -1470,7 +1470,7 @@ __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const
 }
 
 #ifndef GMBE_NI_THR
-#define GMBE_NI_THR 0
+#define GMBE_NI_THR 0  // 1: run_thr out of line -- gh_work -1.5% but dblp +26%, bx +10% (round 2)
 #endif
 #ifndef GMBE_SPLIT_WIDE
 #define GMBE_SPLIT_WIDE 32
@@ -1510,19 +1510,26 @@ __device__ __forceinline__ bool sorted_has(const uint32_t* a, uint32_t n, uint32
   }
   return lo < n && a[lo] == x;
 }
-// Returns false (nothing done) when the job does not fit this tier (no Γ index, too few candidates,
-// more than 64 Q patterns after reduction); the caller then runs it with run_reg.
+// Does a job fit the thread-level tier?  A Γ index (gx) and enough work: adjacency bits beyond one per
+// candidate (a candidate with k = 1 only yields a leaf) -- checked inline by the caller, so the
+// out-of-line run_thr is only entered for jobs it takes.
+__device__ __forceinline__ bool thr_eligible(const Params& P, const TaskCtx& T, const uint32_t* rec) {
+  if (!T.gx) return false;
+  const uint32_t lane = lane_id(), nC = rec[0];
+  uint32_t k = 0;
+  if (lane < nC) k = rec[kHdr + 4 + 4 * lane + (T.W == 2 ? 3 : 2)] - 1u;
+  return warp_sum(k) >= P.thr_min_est;
+}
+// Returns false (nothing done) when the job does not fit this tier (more than 64 Q patterns after
+// reduction); the caller then runs it with run_reg.
 __device__ GMBE_NI_IF(GMBE_NI_THR) bool run_thr(const Params& P, const TaskCtx& T, const uint32_t* rec, uint32_t lmap,
                                                 Acc& A, ThrSmem* ts, unsigned long long* smem, uint32_t* scratch,
                                                 const uint32_t* scratch_end) {
   const uint32_t lane = lane_id();
   const uint32_t nC = rec[0];
-  if (!T.gx) return false;
   const bool w2 = T.W == 2;
   uint4 x = make_uint4(0, 0, 0, 0);
   if (lane < nC) x = ((const uint4*)(rec + kHdr + 4))[lane];
-  // job weight: adjacency bits beyond one per candidate (a candidate with k = 1 only yields a leaf)
-  if (warp_sum(lane < nC ? (w2 ? x.w : x.z) - 1u : 0u) < P.thr_min_est) return false;
   const unsigned long long L0 = ((unsigned long long)rec[kHdr + 1] << 32) | rec[kHdr];
   PH_START(A);
   // the job's candidates (rank order) and universe
@@ -1869,7 +1876,8 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
 #ifndef GMBE_PROFILE
         const unsigned long long n0 = (P.debug & 32) ? A.get(kAcNodes) : 0ull;
 #endif
-        const bool thr = !st && !(P.debug & 16) && run_thr(P, T, reg, lmap, A, ts, smem, reg_scratch, stack_hi);
+        const bool thr = !st && !(P.debug & 16) && thr_eligible(P, T, reg) &&
+                         run_thr(P, T, reg, lmap, A, ts, smem, reg_scratch, stack_hi);
         if (!thr) run_reg(P, T, reg, lmap, A, (RegLevel*)smem, reg_scratch, stack_hi, st, smem);
 #ifndef GMBE_PROFILE
         if (P.debug & 32) {  // path statistics (experiments): jobs / nodes per tier
