@@ -1487,6 +1487,9 @@ __device__ GMBE_NI_IF(GMBE_NI_DONATE_THR) bool donate_thr(const Params& P, const
 #ifndef GMBE_ROOT_CHUNK
 #define GMBE_ROOT_CHUNK 1  // light roots claimed per atomic (opts.root_chunk); >1 measured slower on the heavy-tailed shapes
 #endif
+#ifndef GMBE_WARP_DONATE
+#define GMBE_WARP_DONATE 1  // run_task: warp-level donation of a node's remaining children to idle warps
+#endif
 #ifndef GMBE_THR_DONATE_BURST
 #define GMBE_THR_DONATE_BURST 1  // run_thr: levels donated per check while other warps are hungry (4, 16 measured no better)
 #endif
@@ -1916,9 +1919,16 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     // compacted by this child's Thm 4.1 pass -- go to the queue as one subtask (node (L, R, SR of cur,
     // those candidates)); its children, later sets and prune marks are the ones this warp would have
     // generated, so the tree and every counter are unchanged
-    if (P.donate && !(split_mode && cur == top) && cur[0] >= i + 3 && hungry(P)) {
+    // Only a task's top donates, once (it keeps no remaining children afterwards), and never a top
+    // that is itself a donated piece (node word 1 = 1): without that, a piece is re-donated by every
+    // warp that takes it, copying O(n^2) entries (measured 2-3x slower W/O_PRUNE runs).  A node's
+    // remaining children cannot be split between two warps: Thm 4.1's marks flow from every child to
+    // its later siblings, in order.
+    const uint32_t nrem = cur[0] - (i + 1);
+    if (GMBE_WARP_DONATE && P.donate && cur == top && !split_mode && cur[1] == 0 && nrem >= 4 &&
+        min(cur[2], nrem) * nrem >= 64 && hungry(P)) {
       uint32_t* scr = align4(ch + (r == 2 ? rec_words(T, ch) : 0));
-      const uint32_t n = cur[0] - (i + 1);
+      const uint32_t n = nrem;
       const uint32_t words = kHdr + T.W4 + n * T.E;
       if (scr + words <= stack_hi) {
         const uint32_t* src = cur + kHdr + T.W4 + (size_t)(i + 1) * T.E;
@@ -1926,7 +1936,7 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
         for (uint32_t j = lane; j < n * T.E; j += 32) scr[kHdr + T.W4 + j] = src[j];
         if (lane == 0) {
           scr[0] = n;
-          scr[1] = 0;
+          scr[1] = 1;  // a donated piece: its warp does not donate its top again
           scr[2] = cur[2];
           scr[3] = 0;
           scr[4] = kNone;
