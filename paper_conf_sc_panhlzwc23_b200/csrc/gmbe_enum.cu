@@ -669,14 +669,20 @@ __device__ __forceinline__ bool bsearch_rank(const uint32_t* a, uint32_t n, uint
 }
 
 // Alg 2 L14: is R' == Γ(L')?  Γ(L') = ∩_{u∈L'} N(u) ⊇ R', so maximal iff |Γ(L')| == |R'|.
-// Count over N(u*) for the lowest-degree u* ∈ L', testing the other members of L' in increasing
-// degree order (early exit).  L' = the lc set bits of lmask (W words) over map.
-// scratch: room for next_pow2(lc) 64-bit keys (used when lc > 32).
+// Count over N(u*) for the lowest-degree u* ∈ L' (|Γ(L')| <= deg(u*)), 32 vertices x ∈ N(u*) per
+// step: a cheap necessary filter first (deg(x) >= |L'|), then member-major binary searches of x in
+// the lists of the lowest-degree members while many lanes survive (most x fail at the first ones),
+// then survivor-major verification -- one survivor at a time, its tests against 32 members per step
+// -- once the survivors are few (the members of Γ(L'), i.e. the vertices of R', pass every test:
+// ⌈|L'|/32⌉ steps each instead of |L'| - 1 serial searches).  L' = the lc set bits of lmask (W words)
+// over map.  scratch: room for lc 64-bit keys (used when lc > 32).
 __device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_is_r(const Params& P, const uint32_t* lmask, uint32_t W, const uint32_t* map, uint32_t lc,
                            uint32_t rlen, unsigned long long* scratch, unsigned long long* smem) {
   const uint32_t lane = lane_id();
   const DevGraph& g = P.g;
-  // L' as (deg << 32 | u) keys sorted by degree: lane j holds member j (j < 32)
+  // members as (deg << 32 | begin of N(u)) keys.  lc <= 32: lane j holds the member of j-th lowest
+  // degree.  Wider: all members go to scratch; lane j holds the j-th lowest of the lane-local minima
+  // (the filter members; lane 0 = u*)
   unsigned long long key = ~0ull;
   if (lc <= 32) {
     uint32_t c = 0;  // members gathered so far; the t-th set bit of a word goes to lane c + t
@@ -688,14 +694,13 @@ __device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_is_r(const Params& P, const uint
       const uint32_t src = mine ? __fns(word, 0, lane - c + 1) : 0;
       const uint32_t mine_u = ((word >> lane) & 1u) ? map[w * 32 + lane] : 0u;
       const uint32_t u = __shfl_sync(GMBE_FULL, mine_u, src);
-      if (mine) key = ((unsigned long long)(g.off_u[u + 1] - g.off_u[u]) << 32) | u;
+      if (mine) {
+        const uint32_t b = g.off_u[u];
+        key = ((unsigned long long)(g.off_u[u + 1] - b) << 32) | b;
+      }
       c += nb;
     }
-    key = warp_sort32(key);
   } else {
-    // members -> scratch as (deg << 32 | u), lane-parallel over the mask words; u* = the minimum
-    // (no sort: the wide walk below tests 32 members per step in any order)
-    unsigned long long kmin = ~0ull;
     uint32_t c = 0;
     for (uint32_t wb = 0; wb < W; wb += 32) {
       const uint32_t w = wb + lane;
@@ -709,65 +714,65 @@ __device__ GMBE_NI_IF(GMBE_NI_GAMMA) bool gamma_is_r(const Params& P, const uint
       uint32_t pos = c + inc - nb;
       for (uint32_t x = word; x; x &= x - 1) {
         const uint32_t u = map[w * 32 + __ffs(x) - 1];
-        const unsigned long long kk = ((unsigned long long)(g.off_u[u + 1] - g.off_u[u]) << 32) | u;
+        const uint32_t b = g.off_u[u];
+        const unsigned long long kk = ((unsigned long long)(g.off_u[u + 1] - b) << 32) | b;
         scratch[pos++] = kk;
-        kmin = min(kmin, kk);
+        key = min(key, kk);
       }
       c += __shfl_sync(GMBE_FULL, inc, 31);
     }
-    for (int o = 16; o; o >>= 1) kmin = min(kmin, (unsigned long long)__shfl_xor_sync(GMBE_FULL, kmin, o));
     __syncwarp();
-    key = lane == 0 ? kmin : ~0ull;
   }
+  key = warp_sort32(key);
   const unsigned long long k0 = __shfl_sync(GMBE_FULL, key, 0);
-  const uint32_t d0 = (uint32_t)(k0 >> 32), u0 = (uint32_t)k0;
+  const uint32_t d0 = (uint32_t)(k0 >> 32);
   if (lc == 1 || d0 <= rlen) return d0 == rlen;  // |Γ(L')| <= deg(u*); |L'| = 1: Γ = N(u*)
-  uint32_t mb = 0, md = 0;  // lane j < 32: (begin, degree) of member j's list (|L'| <= 32)
-  if (lc <= 32 && lane < lc) {
-    mb = g.off_u[(uint32_t)key];
-    md = (uint32_t)(key >> 32);
-  }
-  const uint32_t* n0 = g.adj_u + g.off_u[u0];
+  const uint32_t nf = lc <= 32 ? lc : __popc(__ballot_sync(GMBE_FULL, key != ~0ull));  // filter members
+  const uint32_t fb = (uint32_t)key, fd = (uint32_t)(key >> 32);
+  const uint32_t nstep = (lc + 31) >> 5;  // verification steps per survivor
+  const uint32_t* n0 = g.adj_u + (uint32_t)k0;
   uint32_t count = 0;
-  if (lc > 32) {
-    // wide L': one v ∈ N(u*) at a time, lanes test 32 members per step (a member of Γ(L') -- every
-    // vertex of R' -- costs ⌈|L'|/32⌉ steps instead of |L'| - 1; others usually fail in the first)
-    for (uint32_t b = 0; b < d0; b++) {
-      const uint32_t v = __ldg(n0 + b);
+  for (uint32_t b = 0; b < d0; b += 32) {
+    const uint32_t idx = b + lane;
+    bool ok = idx < d0;
+    const uint32_t v = ok ? __ldg(n0 + idx) : 0;
+    if (ok && lc >= 8) ok = g.off_v[v + 1] - g.off_v[v] >= lc;  // a dominator of L' has degree >= |L'|
+    // member-major filter while the survivors would cost more to verify one by one
+    uint32_t j = 1;
+    while (j < nf) {
+      const uint32_t s = __popc(__ballot_sync(GMBE_FULL, ok));
+      if (s * nstep <= nf - j) break;
+      const uint32_t jb = __shfl_sync(GMBE_FULL, fb, j), jd = __shfl_sync(GMBE_FULL, fd, j);
+      if (ok) ok = bsearch_rank(g.adj_u + jb, jd, v);
+      j++;
+    }
+    uint32_t sv = __ballot_sync(GMBE_FULL, ok);
+    if (j >= nf && lc <= 32) {  // every member tested
+      count += __popc(sv);
+      if (count > rlen) return false;
+      continue;
+    }
+    while (sv) {  // survivor-major: 32 members per step, first miss ends the survivor
+      const uint32_t x = __shfl_sync(GMBE_FULL, v, __ffs(sv) - 1);
+      sv &= sv - 1;
       bool all = true;
-      for (uint32_t j0 = 0; j0 < lc && all; j0 += 32) {  // (u* itself passes trivially)
-        const uint32_t j = j0 + lane;
+      for (uint32_t j0 = 0; j0 < lc && all; j0 += 32) {
+        const uint32_t jj = j0 + lane;
         bool in = true;
-        if (j < lc) {
-          const unsigned long long kj = scratch[j];
-          const uint32_t jb = g.off_u[(uint32_t)kj];
-          in = bsearch_rank(g.adj_u + jb, (uint32_t)(kj >> 32), v);
+        if (jj < lc) {
+          uint32_t mb = fb, md = fd;  // lc <= 32: lane jj holds member jj
+          if (lc > 32) {
+            const unsigned long long kj = scratch[jj];
+            mb = (uint32_t)kj;
+            md = (uint32_t)(kj >> 32);
+          }
+          in = bsearch_rank(g.adj_u + mb, md, x);
         }
         all = __all_sync(GMBE_FULL, in);
       }
       count += all;
       if (count > rlen) return false;
     }
-    return count == rlen;
-  }
-  for (uint32_t b = 0; b < d0; b += 32) {
-    const uint32_t idx = b + lane;
-    bool ok = idx < d0;
-    const uint32_t v = ok ? __ldg(n0 + idx) : 0;
-    for (uint32_t j = 1; j < lc && __any_sync(GMBE_FULL, ok); j++) {
-      uint32_t jb, jd;
-      if (j < 32) {
-        jb = __shfl_sync(GMBE_FULL, mb, j);
-        jd = __shfl_sync(GMBE_FULL, md, j);
-      } else {
-        const unsigned long long kj = scratch[j];
-        jb = g.off_u[(uint32_t)kj];
-        jd = (uint32_t)(kj >> 32);
-      }
-      if (ok) ok = bsearch_rank(g.adj_u + jb, jd, v);
-    }
-    count += __popc(__ballot_sync(GMBE_FULL, ok));
-    if (count > rlen) return false;
   }
   return count == rlen;
 }
