@@ -2292,14 +2292,31 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   bool skip = false;
   unsigned long long sr = 0;
   const bool sort_fits = fits(P, (uint32_t*)(sortbuf + next_pow2(max(nocc, 1u))) + 64, M.dyn_end);
-  for (uint32_t b = 0; b < nocc && sort_fits; b += 32) {
+#ifndef GMBE_CLS_UNROLL
+#define GMBE_CLS_UNROLL 2  // occupied-list chunks whose loads are in flight together (memory-level parallelism)
+#endif
+  for (uint32_t b0 = 0; b0 < nocc && sort_fits; b0 += 32 * GMBE_CLS_UNROLL) {
+  uint32_t sq[GMBE_CLS_UNROLL], vq[GMBE_CLS_UNROLL];
+  unsigned long long xq[GMBE_CLS_UNROLL];
+#pragma unroll
+  for (int q = 0; q < GMBE_CLS_UNROLL; q++) sq[q] = b0 + 32 * q + lane < nocc ? occl[b0 + 32 * q + lane] : 0u;
+#pragma unroll
+  for (int q = 0; q < GMBE_CLS_UNROLL; q++) {
+    const bool o = b0 + 32 * q + lane < nocc;
+    vq[q] = o ? (dense ? sq[q] : ldv(keys + sq[q])) : 0u;
+    xq[q] = o ? ldv(vals + sq[q]) : 0ull;
+  }
+#pragma unroll
+  for (int q = 0; q < GMBE_CLS_UNROLL; q++) {
+    const uint32_t b = b0 + 32 * q;
+    if (b >= nocc) break;
     const uint32_t j = b + lane;
     const bool occ = j < nocc;
-    const uint32_t s = occ ? occl[j] : 0;
-    const uint32_t v = occ ? (dense ? s : ldv(keys + s)) : 0;
+    const uint32_t s = sq[q];
+    const uint32_t v = vq[q];
     uint32_t c = 0;
     if (occ) {
-      const unsigned long long x = ldv(vals + s);
+      const unsigned long long x = xq[q];
       c = small ? __popcll(x) : (uint32_t)x;
     }
     const bool isR = occ && c == l;
@@ -2315,6 +2332,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
     const uint32_t bC = __ballot_sync(GMBE_FULL, isC);
     if (isC) sortbuf[nC + __popc(bC & lanemask_lt())] = ((unsigned long long)v << 32) | s;
     nC += __popc(bC);
+  }
   }
   skip = __any_sync(GMBE_FULL, skip);
   if (after != kNone && !skip && sort_fits) skip = earlier_dominator(g, Lr, l, r);
@@ -2358,18 +2376,27 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
         gx[1] = l;
       }
       uint32_t n2 = 0;
-      for (uint32_t b = 0; b < nocc; b += 32) {
-        const uint32_t x = b + lane;
-        const uint32_t slot = x < nocc ? occl[x] : 0u;
-        const unsigned long long row = x < nocc ? ldv(vals + slot) : 0ull;
-        const bool is2 = __popcll(row) >= 2;
-        const uint32_t bal = __ballot_sync(GMBE_FULL, is2);
-        if (is2) {
-          const uint32_t pos = n2 + __popc(bal & lanemask_lt());
-          xrow[pos] = row;
-          xid[pos] = dense ? slot : ldv(keys + slot);
+      for (uint32_t b0 = 0; b0 < nocc; b0 += 32 * GMBE_CLS_UNROLL) {
+        uint32_t sq[GMBE_CLS_UNROLL];
+        unsigned long long rq[GMBE_CLS_UNROLL];
+#pragma unroll
+        for (int q = 0; q < GMBE_CLS_UNROLL; q++) sq[q] = b0 + 32 * q + lane < nocc ? occl[b0 + 32 * q + lane] : 0u;
+#pragma unroll
+        for (int q = 0; q < GMBE_CLS_UNROLL; q++) rq[q] = b0 + 32 * q + lane < nocc ? ldv(vals + sq[q]) : 0ull;
+#pragma unroll
+        for (int q = 0; q < GMBE_CLS_UNROLL; q++) {
+          if (b0 + 32 * q >= nocc) break;
+          const uint32_t slot = sq[q];
+          const unsigned long long row = rq[q];
+          const bool is2 = __popcll(row) >= 2;
+          const uint32_t bal = __ballot_sync(GMBE_FULL, is2);
+          if (is2) {
+            const uint32_t pos = n2 + __popc(bal & lanemask_lt());
+            xrow[pos] = row;
+            xid[pos] = dense ? slot : ldv(keys + slot);
+          }
+          n2 += __popc(bal);
         }
-        n2 += __popc(bal);
       }
       __syncwarp();
       // list lengths: lane j counts universe vertex j (cnt0) and j + 32 (cnt1).  With |X2| <= 64 the
@@ -2530,10 +2557,16 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   }
   // leave the table clean for the next root (the task no longer needs it)
   __syncwarp();
-  for (uint32_t j = lane; j < nocc; j += 32) {
-    const uint32_t s = occl[j];
-    if (!dense) keys[s] = GMBE_EMPTY;
-    vals[s] = 0;
+  for (uint32_t j0 = lane; j0 < nocc; j0 += 32 * GMBE_CLS_UNROLL) {
+    uint32_t sq[GMBE_CLS_UNROLL];
+#pragma unroll
+    for (int q = 0; q < GMBE_CLS_UNROLL; q++) sq[q] = j0 + 32 * q < nocc ? occl[j0 + 32 * q] : kNone;
+#pragma unroll
+    for (int q = 0; q < GMBE_CLS_UNROLL; q++)
+      if (sq[q] != kNone) {
+        if (!dense) keys[sq[q]] = GMBE_EMPTY;
+        vals[sq[q]] = 0;
+      }
   }
   __syncwarp();
   return *top != nullptr;
