@@ -91,7 +91,8 @@ struct Params {
                    // 64 = no suffix-mode roots, 128 = every root in suffix mode, 256 = no dense-mode roots,
                    // 512 = dense mode whenever the table can hold it, 1024 = build the roots only
                    // (timing experiments: no subtree is walked, the result is incomplete),
-                   // 2048 = no register-resident tiny-root build (run_root_tiny)
+                   // 2048 = no register-resident tiny-root build (run_root_tiny), 4096 = no sort-mode
+                   // roots, 8192 = sort mode for every small-universe full-scan root above the smem table
   uint32_t donate;  // dynamic donation to idle warps (donate_reg)
   uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.thr_min)
   uint32_t split_wide;   // wide-universe split threshold on |C|·⌈|L|/32⌉ (opts.split_wide)
@@ -441,6 +442,57 @@ __device__ void warp_radix_pass(const unsigned long long* src, unsigned long lon
     __syncwarp();
     if (j < n && lane == __ffs(peers) - 1) hist[d] += __popc(peers);
     __syncwarp();
+  }
+}
+// the same pass over 32-bit keys, digits of up to 9 bits (hist: 1 << dbits words)
+__device__ void warp_radix_pass32(const uint32_t* src, uint32_t* dst, uint32_t n, uint32_t shift, uint32_t dbits,
+                                  uint32_t* hist) {
+  const uint32_t lane = lane_id(), nb = 1u << dbits;
+  for (uint32_t i = lane; i < nb; i += 32) hist[i] = 0;
+  __syncwarp();
+  for (uint32_t b = 0; b < n; b += 64) {  // two chunks of loads in flight
+    const uint32_t j0 = b + lane, j1 = b + 32 + lane;
+    const uint32_t x0 = j0 < n ? src[j0] : 0u, x1 = j1 < n ? src[j1] : 0u;
+#pragma unroll
+    for (int h = 0; h < 2; h++) {
+      const uint32_t j = h ? j1 : j0;
+      const uint32_t d = j < n ? ((h ? x1 : x0) >> shift) & (nb - 1) : nb;
+      const uint32_t peers = __match_any_sync(GMBE_FULL, d);
+      if (j < n && lane == __ffs(peers) - 1) hist[d] += __popc(peers);
+      __syncwarp();
+    }
+  }
+  const uint32_t per = (nb + 31) / 32;
+  uint32_t loc = 0;
+  for (uint32_t k = 0; k < per; k++)
+    if (lane * per + k < nb) loc += hist[lane * per + k];
+  uint32_t inc = loc;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t t = __shfl_up_sync(GMBE_FULL, inc, o);
+    if (lane >= (uint32_t)o) inc += t;
+  }
+  uint32_t run = inc - loc;
+  __syncwarp();
+  for (uint32_t k = 0; k < per; k++)
+    if (lane * per + k < nb) {
+      const uint32_t c = hist[lane * per + k];
+      hist[lane * per + k] = run;
+      run += c;
+    }
+  __syncwarp();
+  for (uint32_t b = 0; b < n; b += 64) {
+    const uint32_t j0 = b + lane, j1 = b + 32 + lane;
+    const uint32_t x0 = j0 < n ? src[j0] : 0u, x1 = j1 < n ? src[j1] : 0u;
+#pragma unroll
+    for (int h = 0; h < 2; h++) {
+      const uint32_t j = h ? j1 : j0, x = h ? x1 : x0;
+      const uint32_t d = j < n ? (x >> shift) & (nb - 1) : nb;
+      const uint32_t peers = __match_any_sync(GMBE_FULL, d);
+      if (j < n) dst[hist[d] + __popc(peers & lanemask_lt())] = x;
+      __syncwarp();
+      if (j < n && lane == __ffs(peers) - 1) hist[d] += __popc(peers);
+      __syncwarp();
+    }
   }
 }
 // sort n keys in a[0..n) (room for next_pow2(n)); keys above kSmemSort with a scratch tmp[0..n)
@@ -2038,6 +2090,12 @@ __device__ bool earlier_dominator(const DevGraph& g, const uint32_t* Lr, uint32_
 #ifndef GMBE_SUFFIX_MAX_KEEP_L
 #define GMBE_SUFFIX_MAX_KEEP_L 256  // universes up to this size keep a full (dense) scan and their Γ index
 #endif
+#ifndef GMBE_SORT_MIN
+#define GMBE_SORT_MIN 1024  // small-universe roots with at least this many wedges build their rows by sorting
+#endif
+#ifndef GMBE_SORT_MAX
+#define GMBE_SORT_MAX 65536
+#endif
 #ifndef GMBE_SUFFIX_MIN
 #define GMBE_SUFFIX_MIN 8192  // roots with at least this many wedges may scan only later ranks
 #endif
@@ -2225,18 +2283,98 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   unsigned long long* vals = stab ? M.svals : M.vals;
   uint32_t* occl = stab ? M.socc : M.occ;
   const bool small = l <= 64;  // rows (<= 64 bits) straight from the table
+  // Sort mode (B200 addition): a small-universe root with a mid-size wedge scan (the bulk of the
+  // root-construction time on the work-shaped graphs) builds its rows by sorting the wedge keys
+  // (rank << 6 | member index) in a per-root buffer -- LSD radix passes over the rank bits, then one
+  // sweep OR-ing each run of equal rank into its row -- instead of a per-warp table indexed by rank
+  // or by hash.  The buffer (~5 words per wedge) stays in L2, where the dense table's scattered
+  // 8-byte slots (n_v per warp) miss to DRAM.  The occupied ranks come out in rank order, with the
+  // same rows as the tables' (so the same classification, Γ index and candidate order).
+  // Scratch at the end of the warp's dynamic region: keys | keys' | ranks | rows (u64).
+  uint32_t* dyn_end = M.dyn_end;  // the root record and Γ index must end below the sort scratch
+  const uint64_t sort_words = 5ull * r4(scanned) + 32;
+  const bool sorted = small && after == kNone && (!stab || (P.debug & 8192)) && !(P.debug & 4096) &&
+                      (scanned >= GMBE_SORT_MIN || (P.debug & 8192)) && scanned <= GMBE_SORT_MAX &&
+                      M.dyn + 4 * sort_words <= M.dyn_end;
+  uint32_t* s_ck = nullptr;
+  if (sorted) {
+    dyn_end = (uint32_t*)((uintptr_t)(M.dyn_end - sort_words) & ~(uintptr_t)15);
+    s_ck = dyn_end + 2 * r4(scanned);
+    keys = s_ck;
+    vals = (unsigned long long*)(s_ck + r4(scanned));
+  }
   // Dense mode (heavy roots): the warp's table values indexed by rank directly (n_v <= table
   // slots).  Pass 1 is then fire-and-forget atomics (no probing), and the occupied list comes from
   // a scan of the rank range -- in rank order, so the candidates need no sort.
   const uint32_t lo_v = after != kNone ? r + 1 : 0u;
   // The occupied ranks are marked in a per-warp bitmap as well (fire-and-forget atomics), so the
   // scan for them reads (n_v - lo_v)/32 words instead of the whole value range.
-  const bool dense = !stab && g.n_v <= P.tmax && !(P.debug & 256) &&
+  const bool dense = !stab && !sorted && g.n_v <= P.tmax && !(P.debug & 256) &&
                      ((uint64_t)(g.n_v - lo_v) <= (uint64_t)GMBE_DENSE_RATIO * scanned || (P.debug & 512));
+  const bool ident = sorted;  // occupied slot j is entry j of the compact (rank, row) arrays
   PH_START(A);
   // pass 1 (Alg 3 L2-3)
   uint32_t nocc = 0;
-  if (dense) {
+  if (sorted) {
+    uint32_t* kb = dyn_end;
+    uint32_t* kt = dyn_end + r4(scanned);
+    uint32_t wpos = 0;
+    for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
+      if (act) kb[wpos + lane] = (v << 6) | i;
+      wpos += __popc(__ballot_sync(GMBE_FULL, act));
+    });
+    __syncwarp();
+    const uint32_t n = wpos;
+    const uint32_t vb = 32 - __clz(max(g.n_v, 2u) - 1);
+    const uint32_t passes = vb <= 9 ? 1u : vb <= 18 ? 2u : 3u, db = (vb + passes - 1) / passes;
+    for (uint32_t p = 0; p < passes; p++)
+      warp_radix_pass32(p & 1 ? kt : kb, p & 1 ? kb : kt, n, 6 + p * db, db, (uint32_t*)M.sm_sort);
+    const uint32_t* srt = passes & 1 ? kt : kb;
+    __syncwarp();
+    // runs of equal rank -> (rank, row); a run may continue into the next chunk (carry)
+    uint32_t cv = kNone;
+    unsigned long long crow = 0;
+    for (uint32_t b = 0; b < n; b += 32) {
+      const uint32_t j = b + lane;
+      const bool in = j < n;
+      const uint32_t key = in ? srt[j] : 0u;
+      const uint32_t v = in ? key >> 6 : kNone;
+      unsigned long long x = in ? 1ull << (key & 63u) : 0ull;
+      const uint32_t v0 = __shfl_sync(GMBE_FULL, v, 0);
+      if (cv != kNone && v0 != cv && cv != r) {  // the carried run ended with the previous chunk
+        if (lane == 0) {
+          s_ck[nocc] = cv;
+          vals[nocc] = crow;
+        }
+        nocc++;
+      }
+      if (lane == 0 && v == cv) x |= crow;
+      const uint32_t vp = __shfl_up_sync(GMBE_FULL, v, 1);
+      const uint32_t heads = __ballot_sync(GMBE_FULL, lane == 0 || v != vp);
+      const uint32_t ss = 31 - __clz(heads & (lane == 31 ? GMBE_FULL : ((2u << lane) - 1u)));
+#pragma unroll
+      for (uint32_t o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = ((unsigned long long)__shfl_up_sync(GMBE_FULL, (uint32_t)(x >> 32), o) << 32) |
+                                     __shfl_up_sync(GMBE_FULL, (uint32_t)x, o);
+        if (lane >= o && lane - o >= ss) x |= y;
+      }
+      const uint32_t vn = __shfl_down_sync(GMBE_FULL, v, 1);
+      const bool last = b + 32 >= n;
+      const bool end = in && (lane < 31 ? vn != v : last);
+      const bool emit = end && v != r;
+      const uint32_t be = __ballot_sync(GMBE_FULL, emit);
+      if (emit) {
+        const uint32_t q = nocc + __popc(be & lanemask_lt());
+        s_ck[q] = v;
+        vals[q] = x;
+      }
+      nocc += __popc(be);
+      cv = last ? kNone : __shfl_sync(GMBE_FULL, v, 31);
+      crow = ((unsigned long long)__shfl_sync(GMBE_FULL, (uint32_t)(x >> 32), 31) << 32) |
+             __shfl_sync(GMBE_FULL, (uint32_t)x, 31);
+    }
+    __syncwarp();
+  } else if (dense) {
     uint32_t* bits = M.bits;
     for_each_wedge(g, Lr, l, [&](uint32_t i, uint32_t v, bool act) {
       if (act && v != r) {
@@ -2291,7 +2429,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   uint32_t nC = 0, nR = 0, nx2 = 0, sum2 = 0;
   bool skip = false;
   unsigned long long sr = 0;
-  const bool sort_fits = fits(P, (uint32_t*)(sortbuf + next_pow2(max(nocc, 1u))) + 64, M.dyn_end);
+  const bool sort_fits = fits(P, (uint32_t*)(sortbuf + next_pow2(max(nocc, 1u))) + 64, dyn_end);
 #ifndef GMBE_CLS_UNROLL
 #define GMBE_CLS_UNROLL 2  // occupied-list chunks whose loads are in flight together (memory-level parallelism)
 #endif
@@ -2299,7 +2437,8 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   uint32_t sq[GMBE_CLS_UNROLL], vq[GMBE_CLS_UNROLL];
   unsigned long long xq[GMBE_CLS_UNROLL];
 #pragma unroll
-  for (int q = 0; q < GMBE_CLS_UNROLL; q++) sq[q] = b0 + 32 * q + lane < nocc ? occl[b0 + 32 * q + lane] : 0u;
+  for (int q = 0; q < GMBE_CLS_UNROLL; q++)
+    sq[q] = b0 + 32 * q + lane < nocc ? (ident ? b0 + 32 * q + lane : occl[b0 + 32 * q + lane]) : 0u;
 #pragma unroll
   for (int q = 0; q < GMBE_CLS_UNROLL; q++) {
     const bool o = b0 + 32 * q + lane < nocc;
@@ -2350,7 +2489,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   uint32_t* gx = aux;
   uint32_t* rec = align4(aux + (want_aux ? aux_words : 0));
   const uint64_t rec_need = kHdr + W4 + (uint64_t)nC * E;
-  if (sort_fits && !skip && fits(P, rec + rec_need + 64, M.dyn_end)) {
+  if (sort_fits && !skip && fits(P, rec + rec_need + 64, dyn_end)) {
     A.add(kAcRootsRun, 1);
     sr = warp_sum64r(sr) + hv_r;
     unsigned long long sl = 0;
@@ -2380,7 +2519,8 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
         uint32_t sq[GMBE_CLS_UNROLL];
         unsigned long long rq[GMBE_CLS_UNROLL];
 #pragma unroll
-        for (int q = 0; q < GMBE_CLS_UNROLL; q++) sq[q] = b0 + 32 * q + lane < nocc ? occl[b0 + 32 * q + lane] : 0u;
+        for (int q = 0; q < GMBE_CLS_UNROLL; q++)
+          sq[q] = b0 + 32 * q + lane < nocc ? (ident ? b0 + 32 * q + lane : occl[b0 + 32 * q + lane]) : 0u;
 #pragma unroll
         for (int q = 0; q < GMBE_CLS_UNROLL; q++) rq[q] = b0 + 32 * q + lane < nocc ? ldv(vals + sq[q]) : 0ull;
 #pragma unroll
@@ -2458,7 +2598,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
       // root node record: candidates in rank order (Alg 2 L6 "smallest first")
       __syncwarp();
       PH_STOP(A, 3);
-      if (!dense)  // dense mode: occupied list (and so the candidates) already in rank order
+      if (!dense && !sorted)  // dense / sort mode: occupied list (and so the candidates) already in rank order
         warp_sort_keys(sortbuf, nC, M.sm_sort, (unsigned long long*)rec, 32 - __clz(max(g.n_v, 2u) - 1));
       PH_STOP(A, 2);
       uint32_t* ent = rec + kHdr + W4;
@@ -2557,7 +2697,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   }
   // leave the table clean for the next root (the task no longer needs it)
   __syncwarp();
-  for (uint32_t j0 = lane; j0 < nocc; j0 += 32 * GMBE_CLS_UNROLL) {
+  for (uint32_t j0 = lane; j0 < (sorted ? 0u : nocc); j0 += 32 * GMBE_CLS_UNROLL) {  // (sort mode: scratch)
     uint32_t sq[GMBE_CLS_UNROLL];
 #pragma unroll
     for (int q = 0; q < GMBE_CLS_UNROLL; q++) sq[q] = j0 + 32 * q < nocc ? occl[j0 + 32 * q] : kNone;

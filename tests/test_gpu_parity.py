@@ -411,6 +411,37 @@ def test_dense_mode_roots(gmbe, dense_case):
             _same(_run(gmbe, nu, nv, e, debug=dbg), o)
 
 
+def test_sort_mode_roots(gmbe, dense_case):
+    """Sort-mode roots (rows built by radix-sorting the wedge keys rank << 6 | member, runs of equal
+    rank OR-ed into rows; no per-warp table) forced on every small-universe full-scan root
+    (debug 8192), and switched off (debug 4096): the canonical tree, sets and counters."""
+    nu, nv, e, o = dense_case
+    g = gmbe.load(nu, nv, e)
+    try:
+        for dbg in (8192, 8192 | 16, 4096):
+            r = g.enumerate(records=True, debug=dbg)
+            _same(r, o)
+            assert r.bicliques == sorted(o.bicliques), dbg
+        r = g.enumerate(records=True, debug=8192, bound_height=1, bound_size=1)
+        _same(r, o)
+    finally:
+        g.free()
+    rng = np.random.default_rng(79)
+    for it in range(60):
+        nu, nv, e = _rand_graph(rng, nmax=14)
+        o = oracle.oracle_mbe(nu, nv, e, records=True)
+        r = _run(gmbe, nu, nv, e, records=True, debug=8192)
+        _same(r, o)
+        assert r.bicliques == sorted(o.bicliques)
+    # many wedges per root over a 64-bit universe, rows across the 32-bit boundary, ranks > 2^9
+    for it in range(3):
+        nu, nv = int(rng.integers(2500, 3500)), int(rng.integers(600, 1400))
+        e = np.argwhere(rng.random((nu, nv)) < 0.015).astype(np.uint32)
+        o = oracle.oracle_mbe(nu, nv, e)
+        for dbg in (8192, 4096, 0):
+            _same(_run(gmbe, nu, nv, e, debug=dbg), o)
+
+
 # ---------------------------------------------------------------- streaming output (N2)
 def _stream_all(g, **kw):
     got = []
