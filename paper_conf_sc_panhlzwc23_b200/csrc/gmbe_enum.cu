@@ -97,6 +97,7 @@ struct Params {
   uint32_t thr_min_est;  // run_thr tier threshold on Σ_c (k_c - 1) (opts.thr_min)
   uint32_t split_wide;   // wide-universe split threshold on |C|·⌈|L|/32⌉ (opts.split_wide)
   uint32_t chunk, chunk_from;  // root claims: `chunk` issue positions per atomic past position chunk_from
+  uint32_t sort_min;           // sort-mode roots from this many wedges (kNone: off for this call)
   unsigned long long* timeline;  // profiling: [cursor, then (smid<<56|kind<<48|root), t0, t1, info]*
   uint64_t timeline_cap;
   unsigned long long* shared_cursor;  // N1: root cursor shared across GPUs / processes (opts.root_cursor)
@@ -2294,7 +2295,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   uint32_t* dyn_end = M.dyn_end;  // the root record and Γ index must end below the sort scratch
   const uint64_t sort_words = 5ull * r4(scanned) + 32;
   const bool sorted = small && after == kNone && (!stab || (P.debug & 8192)) && !(P.debug & 4096) &&
-                      (scanned >= GMBE_SORT_MIN || (P.debug & 8192)) && scanned <= GMBE_SORT_MAX &&
+                      (scanned >= P.sort_min || (P.debug & 8192)) && scanned <= GMBE_SORT_MAX &&
                       M.dyn + 4 * sort_words <= M.dyn_end;
   uint32_t* s_ck = nullptr;
   if (sorted) {
@@ -3281,6 +3282,13 @@ static int enumerate_once(const gmbe_graph* G, const gmbe_opts& o, gmbe_sink_fn 
   // per atomic), a warp claims root_chunk consecutive positions per atomic (default 1, <= 32)
   P.chunk = o.root_chunk ? std::min<uint32_t>(o.root_chunk, 32u) : GMBE_ROOT_CHUNK;
   P.chunk_from = P.n_roots / 8;
+  // Sort-mode roots trade per-root latency (two radix passes and a grouping sweep instead of one table
+  // pass) for L2-resident traffic: they pay when the root builds of every resident warp contend for
+  // DRAM (a full graph on one GPU: gh_work 14.8 -> 14.45 ms), not when a shard leaves the GPU
+  // latency-bound (1/8 cost parts of gh_work: mean part 2.91 -> 3.31 ms).  On only while the call
+  // has many roots per resident warp (and not under the N1 shared cursor, whose issue list is the
+  // whole graph's while this GPU takes only its share of it).
+  P.sort_min = !o.root_cursor && (uint64_t)P.n_roots >= 8ull * nwarps ? GMBE_SORT_MIN : kNone;
   P.split_wide = o.split_wide ? o.split_wide : GMBE_SPLIT_WIDE;
   P.timeline = (unsigned long long*)o.timeline;
   P.timeline_cap = o.timeline_cap;
