@@ -1131,10 +1131,9 @@ __device__ int gen_child_small(const Params& P, const TaskCtx& T, uint32_t* par,
   const uint32_t rlen = par[5] + 1 + r_abs;
   PH_STOP(A, 4);
   bool maximal;
-  if (lc == 1) {  // Γ({u}) = N(u)
+  if (lc == 1) {  // Γ({u}) = N(u); the universe vertices' degrees are lane-resident (small_task_init)
     const uint32_t j = __ffsll(lm) - 1;
-    const uint32_t u = T.map[j];
-    maximal = P.g.off_u[u + 1] - P.g.off_u[u] == rlen;
+    maximal = __shfl_sync(GMBE_FULL, j < 32 ? T.dg0 : T.dg1, j & 31) == rlen;
   } else if (T.gx) {
     maximal = gamma_gx_small(T, lm, rlen);
   } else {
@@ -1348,9 +1347,9 @@ __device__ GMBE_NI_IF(GMBE_NI_REG) void run_reg(const Params& P, const TaskCtx& 
     A.add(kAcAbytes, 4ull * (lc + __reduce_add_sync(GMBE_FULL, inl ? kp : 0u)));
     const uint32_t rl = rlen + 1 + __popc(ab);
     bool maximal;
-    if (lc == 1) {
-      const uint32_t u = T.map[__ffsll(lp) - 1];
-      maximal = P.g.off_u[u + 1] - P.g.off_u[u] == rl;
+    if (lc == 1) {  // (degrees lane-resident, small_task_init)
+      const uint32_t j = __ffsll(lp) - 1;
+      maximal = __shfl_sync(GMBE_FULL, j < 32 ? T.dg0 : T.dg1, j & 31) == rl;
     } else if (T.gx) {
       maximal = gamma_gx_small(T, lp, rl);
     } else {
