@@ -2294,6 +2294,7 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   uint32_t* dyn_end = M.dyn_end;  // the root record and Γ index must end below the sort scratch
   const uint64_t sort_words = 5ull * r4(scanned) + 32;
   const bool sorted = small && after == kNone && (!stab || (P.debug & 8192)) && !(P.debug & 4096) &&
+                      g.n_v < (1u << 26) &&  // keys rank << 6 | member must fit 32 bits
                       (scanned >= P.sort_min || (P.debug & 8192)) && scanned <= GMBE_SORT_MAX &&
                       M.dyn + 4 * sort_words <= M.dyn_end;
   uint32_t* s_ck = nullptr;
