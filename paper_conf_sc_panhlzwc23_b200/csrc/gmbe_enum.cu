@@ -3288,7 +3288,11 @@ static int enumerate_once(const gmbe_graph* G, const gmbe_opts& o, gmbe_sink_fn 
   // latency-bound (1/8 cost parts of gh_work: mean part 2.91 -> 3.31 ms).  On only while the call
   // has many roots per resident warp (and not under the N1 shared cursor, whose issue list is the
   // whole graph's while this GPU takes only its share of it).
-  P.sort_min = !o.root_cursor && (uint64_t)P.n_roots >= 8ull * nwarps ? GMBE_SORT_MIN : kNone;
+  const bool saturated = !o.root_cursor && (uint64_t)P.n_roots >= 8ull * nwarps;
+  P.sort_min = saturated ? GMBE_SORT_MIN : kNone;
+  // Split threshold (B2): a saturated call splits a little less (bound_size 550: gh_work 14.1 -> 13.9 ms
+  // at N=1), a shard more (550 made 1/8 cost parts of gh_work 2.85 -> 2.98 ms mean): same rule as above
+  if (!o.bound_size) P.bound_size = saturated ? 550 : 500;
   P.split_wide = o.split_wide ? o.split_wide : GMBE_SPLIT_WIDE;
   P.timeline = (unsigned long long*)o.timeline;
   P.timeline_cap = o.timeline_cap;
