@@ -2088,7 +2088,7 @@ __device__ bool earlier_dominator(const DevGraph& g, const uint32_t* Lr, uint32_
 #define GMBE_DENSE_RATIO 32  // dense root tables when the scanned rank range <= this x the wedges
 #endif
 #ifndef GMBE_SUFFIX_MAX_KEEP_L
-#define GMBE_SUFFIX_MAX_KEEP_L 256  // universes up to this size keep a full (dense) scan and their Γ index
+#define GMBE_SUFFIX_MAX_KEEP_L 1024  // universes up to this size keep a full (dense) scan and their Γ index (256: bx_work 25.45 ms, 1024: 22.95)
 #endif
 #ifndef GMBE_SORT_MIN
 #define GMBE_SORT_MIN 1024  // small-universe roots with at least this many wedges build their rows by sorting
