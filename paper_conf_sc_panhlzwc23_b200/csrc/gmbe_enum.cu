@@ -2259,7 +2259,10 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
       sp += du - upper_rank(g.adj_u + ub, du, r);
     }
     sp = warp_sum(sp);
-    if (4ull * sp < wedges) {
+#ifndef GMBE_SUFFIX_RATIO
+#define GMBE_SUFFIX_RATIO 4  // suffix mode when fewer than 1/ratio of the wedges reach later ranks
+#endif
+    if ((unsigned long long)GMBE_SUFFIX_RATIO * sp < wedges) {
       after = r;
       scanned = sp;
     }
@@ -3233,7 +3236,10 @@ static int enumerate_once(const gmbe_graph* G, const gmbe_opts& o, gmbe_sink_fn 
   P.hu_side = g.swapped ? 1 : 0;
   P.arena = (uint32_t*)W.arena;
   P.arena_words = arena_words;
-  P.col_budget = W.dyn / 2;
+#ifndef GMBE_COL_BUDGET_PCT
+#define GMBE_COL_BUDGET_PCT 50  // a root's Γ index may take this % of the warp's dynamic region
+#endif
+  P.col_budget = W.dyn * GMBE_COL_BUDGET_PCT / 100;
   P.tmax = (uint32_t)tmax;
   P.omax = (uint32_t)omax;
   P.bmax = (uint32_t)bmax_use;
