@@ -1982,8 +1982,11 @@ __device__ void run_task(const Params& P, const TaskCtx& T, uint32_t* top, uint3
     // remaining children cannot be split between two warps: Thm 4.1's marks flow from every child to
     // its later siblings, in order.
     const uint32_t nrem = cur[0] - (i + 1);
+#ifndef GMBE_WARP_DONATE_MIN
+#define GMBE_WARP_DONATE_MIN 64  // warp-level donation of a top's remaining children: min(|L|, n) * n at least this
+#endif
     if (GMBE_WARP_DONATE && P.donate && cur == top && !split_mode && cur[1] == 0 && nrem >= 4 &&
-        min(cur[2], nrem) * nrem >= 64 && hungry(P)) {
+        min(cur[2], nrem) * nrem >= GMBE_WARP_DONATE_MIN && hungry(P)) {
       uint32_t* scr = align4(ch + (r == 2 ? rec_words(T, ch) : 0));
       const uint32_t n = nrem;
       const uint32_t words = kHdr + T.W4 + n * T.E;
