@@ -2252,22 +2252,30 @@ __device__ GMBE_NI_IF(GMBE_NI_ROOT) bool run_root(const Params& P, uint32_t r, u
   uint32_t after = kNone, scanned = wedges;
   if (P.debug & 128) {  // tests: every root in suffix mode
     after = r;
-  } else if (wedges >= GMBE_SUFFIX_MIN && !(P.debug & 64) &&
-             // a small universe that a dense full scan can afford keeps its Γ index (thread tier)
-             !(l <= GMBE_SUFFIX_MAX_KEEP_L && g.n_v <= P.tmax && (uint64_t)g.n_v <= 16ull * wedges &&
-               !(P.debug & 256))) {
-    uint32_t sp = 0;
-    for (uint32_t j = lane; j < l; j += 32) {
-      const uint32_t u = Lr[j], ub = g.off_u[u], du = g.off_u[u + 1] - ub;
-      sp += du - upper_rank(g.adj_u + ub, du, r);
-    }
-    sp = warp_sum(sp);
+  } else if (wedges >= GMBE_SUFFIX_MIN && !(P.debug & 64)) {
+    // a universe that a dense full scan can afford keeps its Γ index (thread tier / Γ columns): up to
+    // 256 vertices always, up to GMBE_SUFFIX_MAX_KEEP_L when enough wedges reach later ranks that
+    // the subtree is likely to be worked (B5; bx-shaped roots of 300-1,000 vertices with ~1,000 later
+    // wedges vs GH-shaped hubs with ~100)
+    const bool keepable = l <= GMBE_SUFFIX_MAX_KEEP_L && g.n_v <= P.tmax && (uint64_t)g.n_v <= 16ull * wedges &&
+                          !(P.debug & 256);
+    if (!keepable || l > 256) {
+      uint32_t sp = 0;
+      for (uint32_t j = lane; j < l; j += 32) {
+        const uint32_t u = Lr[j], ub = g.off_u[u], du = g.off_u[u + 1] - ub;
+        sp += du - upper_rank(g.adj_u + ub, du, r);
+      }
+      sp = warp_sum(sp);
 #ifndef GMBE_SUFFIX_RATIO
 #define GMBE_SUFFIX_RATIO 4  // suffix mode when fewer than 1/ratio of the wedges reach later ranks
 #endif
-    if ((unsigned long long)GMBE_SUFFIX_RATIO * sp < wedges) {
-      after = r;
-      scanned = sp;
+#ifndef GMBE_SUFFIX_KEEP_SP
+#define GMBE_SUFFIX_KEEP_SP 512
+#endif
+      if ((unsigned long long)GMBE_SUFFIX_RATIO * sp < wedges && !(keepable && sp >= GMBE_SUFFIX_KEEP_SP)) {
+        after = r;
+        scanned = sp;
+      }
     }
   }
   if (after != kNone && (P.debug & 128)) {
